@@ -1,0 +1,612 @@
+/*
+ * oracle.c -- PreScaler CPU ORACLE.  TEST INFRASTRUCTURE ONLY: only tests/,
+ * __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference leg
+ * may load this.  It shares no code with the CUDA path.
+ *
+ * Plain, slow, single-threaded C written to be checked against the paper by
+ * eye.  Build: gcc -O2 -ffp-contract=off -fno-fast-math (no FMA contraction,
+ * no FTZ/DAZ), x86-64 SSE arithmetic (float ops are IEEE single, double ops
+ * IEEE double).  Every narrowing conversion goes through the software
+ * bit-manipulation converter below, never an FPU conversion instruction.
+ *
+ * What it computes (readings listed in DESIGN.md):
+ *   a1 config decode   ("(1+#Conv_Types)^N", order P:293)
+ *   a2 input conversion of every memory object to its assigned precision
+ *      (device-side conversion, Fig. 3c; memory-object scaling P:55-57)
+ *   a3 the precision-scaled application statements (readings R1-R5)
+ *   a4 back-conversion of the outputs to their original type
+ *   a5 mean-relative-error quality vs the fp64 run and the TOQ test
+ *      "Accuracy < TOQ -> fail" (Alg. 1 line 10)
+ *
+ * Pins (tests/test_oracle_*.py): F16C hardware + numpy over all 2^32 fp32
+ * inputs, numpy + AVX512-FP16 on fp64 inputs, paper fixed points
+ * (tests/golden/), numpy float64 textbook results for every app, exact-integer
+ * invariants for the reduction orders, closed forms for the quality metric.
+ */
+#include "oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ===================================================================== */
+/* c-1: software IEEE-754 converter                                      */
+/* ===================================================================== */
+
+typedef struct { int ebits, mbits, bias; } fmt_t;
+/* index = precision code: f64, f32, f16 */
+static const fmt_t FMT[3] = { {11, 52, 1023}, {8, 23, 127}, {5, 10, 15} };
+
+/* number of significant bits of v (0 for v == 0) */
+static int bitlen64(uint64_t v) { return v ? 64 - __builtin_clzll(v) : 0; }
+
+/* Reading #5 (R-NaN): canonical NaN = every bit set except the sign bit. */
+static uint64_t canonical_nan(const fmt_t *d) {
+  int w = 1 + d->ebits + d->mbits;
+  return (w == 64) ? 0x7FFFFFFFFFFFFFFFull : ((1ull << (w - 1)) - 1);
+}
+
+uint64_t oracle_convert_bits(uint64_t x, int st, int dt) {
+  const fmt_t *s = &FMT[st], *d = &FMT[dt];
+  int sw = 1 + s->ebits + s->mbits, dw = 1 + d->ebits + d->mbits;
+  uint64_t sign = (x >> (sw - 1)) & 1u;
+  uint64_t e = (x >> s->mbits) & ((1ull << s->ebits) - 1);
+  uint64_t f = x & ((1ull << s->mbits) - 1);
+  uint64_t emax_s = (1ull << s->ebits) - 1, emax_d = (1ull << d->ebits) - 1;
+  uint64_t dsign = sign << (dw - 1);
+  uint64_t S, K;
+  int xexp, E, q, r, emin_d;
+
+  /* step 2: inf / NaN */
+  if (e == emax_s) {
+    if (f == 0) return dsign | (emax_d << d->mbits);
+    return canonical_nan(d);
+  }
+  /* step 3: signed zero */
+  if (e == 0 && f == 0) return dsign;
+  /* step 4: value = S * 2^xexp */
+  if (e == 0) { S = f; xexp = 1 - s->bias - s->mbits; }
+  else        { S = f | (1ull << s->mbits); xexp = (int)e - s->bias - s->mbits; }
+  /* step 5: unbiased exponent of the leading bit */
+  E = bitlen64(S) - 1 + xexp;
+  /* step 7.1: destination quantum exponent (subnormal floor emin_d) */
+  emin_d = 1 - d->bias;
+  q = (E > emin_d ? E : emin_d) - d->mbits;
+  r = q - xexp;
+  if (r <= 0) {
+    K = S << (-r);                 /* exact (widening, or narrowing w/o loss) */
+  } else if (r > bitlen64(S)) {
+    K = 0;                         /* below half of the smallest quantum      */
+  } else {
+    /* step 7.4: round to nearest, ties to even */
+    uint64_t rem = S & ((1ull << r) - 1), half = 1ull << (r - 1);
+    K = S >> r;
+    if (rem > half || (rem == half && (K & 1u))) K++;
+  }
+  if (K == 0) return dsign;
+  /* step 8: encode */
+  if (K >= (1ull << d->mbits)) {
+    int64_t biased = (int64_t)q + d->mbits + d->bias;
+    if (K == (1ull << (d->mbits + 1))) { K >>= 1; biased++; }
+    if (biased >= (int64_t)emax_d) return dsign | (emax_d << d->mbits);   /* overflow -> inf */
+    return dsign | ((uint64_t)biased << d->mbits) | (K - (1ull << d->mbits));
+  }
+  return dsign | K;                /* subnormal (q == emin_d - mbits) */
+}
+
+static uint64_t load_bits(const void *p, int t, size_t i) {
+  switch (t) {
+    case OR_F64: { uint64_t b; memcpy(&b, (const char *)p + 8 * i, 8); return b; }
+    case OR_F32: { uint32_t b; memcpy(&b, (const char *)p + 4 * i, 4); return b; }
+    default:     { uint16_t b; memcpy(&b, (const char *)p + 2 * i, 2); return b; }
+  }
+}
+static void store_bits(void *p, int t, size_t i, uint64_t b) {
+  switch (t) {
+    case OR_F64: memcpy((char *)p + 8 * i, &b, 8); break;
+    case OR_F32: { uint32_t v = (uint32_t)b; memcpy((char *)p + 4 * i, &v, 4); break; }
+    default:     { uint16_t v = (uint16_t)b; memcpy((char *)p + 2 * i, &v, 2); break; }
+  }
+}
+
+int oracle_convert(const void *src, int st, void *dst, int dt, size_t n) {
+  size_t i;
+  if (st < 0 || st > 2 || dt < 0 || dt > 2) return 1;
+  if (n && (!src || !dst)) return 1;
+  for (i = 0; i < n; i++) {
+    uint64_t b = load_bits(src, st, i);
+    store_bits(dst, dt, i, st == dt ? b : oracle_convert_bits(b, st, dt));
+  }
+  return 0;
+}
+
+static double bits_to_double(uint64_t b) { double d; memcpy(&d, &b, 8); return d; }
+static uint64_t double_to_bits(double d) { uint64_t b; memcpy(&b, &d, 8); return b; }
+static uint32_t float_to_bits(float f) { uint32_t b; memcpy(&b, &f, 4); return b; }
+static float bits_to_float(uint32_t b) { float f; memcpy(&f, &b, 4); return f; }
+
+/* exact widening of element i of a buffer of type t to double */
+static double widen(const void *p, int t, size_t i) {
+  uint64_t b = load_bits(p, t, i);
+  return bits_to_double(t == OR_F64 ? b : oracle_convert_bits(b, t, OR_F64));
+}
+
+/* ===================================================================== */
+/* c-5: quality                                                          */
+/* ===================================================================== */
+
+void oracle_quality_accumulate(const void *out, int ot, const double *ref, size_t n,
+                               double *sum_e, double *max_rel, uint64_t *nonfinite) {
+  size_t i;
+  for (i = 0; i < n; i++) {
+    double o = widen(out, ot, i), r = ref[i], e, rel;
+    if (!isfinite(o)) (*nonfinite)++;
+    if (o == r) { e = 0.0; rel = 0.0; }
+    else if (!isfinite(o) || !isfinite(r) || r == 0.0) { e = 1.0; rel = INFINITY; }
+    else { rel = fabs(o - r) / fabs(r); e = rel < 1.0 ? rel : 1.0; }
+    *sum_e = *sum_e + e;
+    if (rel > *max_rel) *max_rel = rel;
+  }
+}
+
+int oracle_quality(const void *out, int ot, const double *ref, size_t n,
+                   oracle_quality_result *res) {
+  double s = 0.0, mx = 0.0;
+  uint64_t nf = 0;
+  if (!res || ot < 0 || ot > 2) return 1;
+  oracle_quality_accumulate(out, ot, ref, n, &s, &mx, &nf);
+  res->n = n;
+  res->mean_rel = n ? s / (double)n : 0.0;
+  res->quality = 1.0 - res->mean_rel;
+  res->max_rel = mx;
+  res->nonfinite = nf;
+  return 0;
+}
+
+/* ===================================================================== */
+/* c-2: configuration codec                                              */
+/* ===================================================================== */
+
+int oracle_config_decode(int m, uint64_t id, int *prec) {
+  int i;
+  uint64_t space = 1;
+  for (i = 0; i < m; i++) space *= 3;
+  if (m <= 0 || id >= space || !prec) return 1;
+  for (i = 0; i < m; i++) { prec[i] = (int)(id % 3); id /= 3; }
+  return 0;
+}
+
+int oracle_config_encode(int m, const int *prec, uint64_t *id) {
+  int i;
+  uint64_t v = 0, w = 1;
+  if (m <= 0 || !prec || !id) return 1;
+  for (i = 0; i < m; i++) {
+    if (prec[i] < 0 || prec[i] > 2) return 1;
+    v += (uint64_t)prec[i] * w;
+    w *= 3;
+  }
+  *id = v;
+  return 0;
+}
+
+/* ===================================================================== */
+/* R1/R2/R4: objects and arithmetic "in T"                               */
+/* ===================================================================== */
+
+typedef struct { int type; size_t n; void *p; } obj_t;
+
+static size_t tsize(int t) { return t == OR_F64 ? 8 : (t == OR_F32 ? 4 : 2); }
+
+/* R1: load = exact widening of the stored element */
+static double ld(const obj_t *o, size_t i) { return widen(o->p, o->type, i); }
+
+/* R1: store = RNE from the compute type T to the object's precision.  The
+ * value v is exactly representable in T. */
+static void st(obj_t *o, size_t i, double v, int T) {
+  uint64_t b;
+  if (o->type == OR_F64) { ((double *)o->p)[i] = v; return; }
+  if (T == OR_F64) b = oracle_convert_bits(double_to_bits(v), OR_F64, o->type);
+  else if (o->type == OR_F32) b = float_to_bits((float)v);        /* exact: v is f32 */
+  else b = oracle_convert_bits(float_to_bits((float)v), OR_F32, OR_F16);
+  store_bits(o->p, o->type, i, b);
+}
+
+/* R2: T = widest of the touched objects, floored at f32 (code 0 = widest) */
+static int W2(int a, int b) { int t = a < b ? a : b; return t < OR_F32 ? t : OR_F32; }
+static int W3(int a, int b, int c) { return W2(W2(a, b), c); }
+
+/* R4: single correctly rounded IEEE operations in T.  Operands are exactly
+ * representable in T, so the (float) casts below are exact. */
+static double t_add(int T, double a, double b) {
+  return T == OR_F64 ? a + b : (double)((float)a + (float)b);
+}
+static double t_sub(int T, double a, double b) {
+  return T == OR_F64 ? a - b : (double)((float)a - (float)b);
+}
+static double t_mul(int T, double a, double b) {
+  return T == OR_F64 ? a * b : (double)((float)a * (float)b);
+}
+static double t_div(int T, double a, double b) {
+  return T == OR_F64 ? a / b : (double)((float)a / (float)b);
+}
+static double t_fma(int T, double a, double b, double c) {
+  return T == OR_F64 ? fma(a, b, c) : (double)fmaf((float)a, (float)b, (float)c);
+}
+static double t_sqrt(int T, double a) {
+  return T == OR_F64 ? sqrt(a) : (double)sqrtf((float)a);
+}
+/* R2: scalars are RNE-rounded from their fp64 literal to T */
+static double t_lit(int T, double lit) {
+  if (T == OR_F64) return lit;
+  return (double)bits_to_float((uint32_t)oracle_convert_bits(double_to_bits(lit), OR_F64, OR_F32));
+}
+
+/* ===================================================================== */
+/* R3 / R5: canonical reduction orders                                   */
+/* ===================================================================== */
+
+/* R3: C_ij-style contraction: acc <- fma(a_k, b_k, acc) from +0, k ascending.
+ * a(k) = A[ai + k*ask], b(k) = B[bi + k*bsk]. */
+static double dot_chain(int T, const obj_t *A, size_t ai, size_t ask,
+                        const obj_t *B, size_t bi, size_t bsk, size_t K) {
+  double acc = 0.0;
+  size_t k;
+  for (k = 0; k < K; k++) acc = t_fma(T, ld(A, ai + k * ask), ld(B, bi + k * bsk), acc);
+  return acc;
+}
+
+/* R5 row-dot: y = sum_j A[row, j] x_j for a row of length n.  Lane l of 32
+ * owns the 16-byte chunks c = t*32 + l (V = 16 / sizeof(stored A) elements
+ * each) and runs an fma chain over them (t ascending, then v ascending).
+ * Lanes then combine by xor butterfly with offsets 16,8,4,2,1 as a + partner. */
+static double rowdot(int T, const obj_t *A, size_t row0, size_t n, const obj_t *x) {
+  double lane[ORACLE_ROWDOT_LANES], nxt[ORACLE_ROWDOT_LANES];
+  size_t V = 16 / tsize(A->type), nchunks = (n + V - 1) / V, c, v;
+  int l, off;
+  for (l = 0; l < ORACLE_ROWDOT_LANES; l++) lane[l] = 0.0;
+  for (c = 0; c < nchunks; c++) {
+    l = (int)(c % ORACLE_ROWDOT_LANES);
+    for (v = 0; v < V && c * V + v < n; v++) {
+      size_t j = c * V + v;
+      lane[l] = t_fma(T, ld(A, row0 + j), ld(x, j), lane[l]);
+    }
+  }
+  for (off = ORACLE_ROWDOT_LANES / 2; off >= 1; off >>= 1) {
+    for (l = 0; l < ORACLE_ROWDOT_LANES; l++) nxt[l] = t_add(T, lane[l], lane[l ^ off]);
+    memcpy(lane, nxt, sizeof(lane));
+  }
+  return lane[0];
+}
+
+/* R5 column-sum: z_j = sum_i A_ij w_i.  Rows are split into chunks of
+ * ORACLE_COLSUM_CHUNK; each chunk runs an fma chain from +0 (i ascending);
+ * the chunk partials are added in ascending chunk order (total = p_0 first).
+ * mode 0: term fma(A_ij, w_i, p); mode 1: p + A_ij (w ignored);
+ * mode 2: d = A_ij - mu_j, fma(d, d, p) (mu = w, indexed by column). */
+static double colsum(int T, const obj_t *A, size_t nrows, size_t ncols, size_t j,
+                     const obj_t *w, int mode) {
+  double total = 0.0, p;
+  size_t c0, i;
+  for (c0 = 0; c0 < nrows; c0 += ORACLE_COLSUM_CHUNK) {
+    size_t c1 = c0 + ORACLE_COLSUM_CHUNK < nrows ? c0 + ORACLE_COLSUM_CHUNK : nrows;
+    p = 0.0;
+    for (i = c0; i < c1; i++) {
+      double a = ld(A, i * ncols + j);
+      if (mode == 0) p = t_fma(T, a, ld(w, i), p);
+      else if (mode == 1) p = t_add(T, p, a);
+      else { double d = t_sub(T, a, ld(w, j)); p = t_fma(T, d, d, p); }
+    }
+    total = (c0 == 0) ? p : t_add(T, total, p);
+  }
+  return total;
+}
+
+/* ===================================================================== */
+/* c-4: applications                                                     */
+/* ===================================================================== */
+
+typedef struct {
+  const char *kind;
+  int nobj, ndims_full;
+  const char *names[8];
+  int roles[8];
+  int outputs[8];
+} app_def_t;
+
+/* object order = configuration-id digit order (c-2) */
+static const app_def_t APPS[] = {
+  {"gemm", 3, 3, {"A", "B", "C"}, {0, 0, 2}, {0, 0, 1}},
+  {"2mm", 5, 4, {"A", "B", "C", "D", "E"}, {0, 0, 3, 0, 1}, {0, 0, 0, 0, 1}},
+  {"3mm", 7, 5, {"A", "B", "C", "D", "E", "F", "G"}, {0, 0, 0, 0, 3, 3, 1}, {0, 0, 0, 0, 0, 0, 1}},
+  {"atax", 4, 2, {"A", "x", "y", "tmp"}, {0, 0, 1, 3}, {0, 0, 1, 0}},
+  {"bicg", 5, 2, {"A", "r", "s", "p", "q"}, {0, 0, 1, 0, 1}, {0, 0, 1, 0, 1}},
+  {"gesummv", 5, 1, {"A", "B", "x", "y", "tmp"}, {0, 0, 0, 1, 3}, {0, 0, 0, 1, 0}},
+  {"corr", 4, 2, {"data", "mean", "stddev", "symmat"}, {2, 3, 3, 1}, {0, 0, 0, 1}},
+  {"covar", 3, 2, {"data", "mean", "symmat"}, {2, 3, 1}, {0, 0, 1}},
+};
+
+static const app_def_t *find_app(const char *kind) {
+  size_t i;
+  if (!kind) return NULL;
+  for (i = 0; i < sizeof(APPS) / sizeof(APPS[0]); i++)
+    if (strcmp(APPS[i].kind, kind) == 0) return &APPS[i];
+  return NULL;
+}
+
+/* expand dims: ndims == 1 means every dimension equals dims[0] */
+static int full_dims(const app_def_t *a, const int64_t *dims, int ndims, int64_t *d) {
+  int i;
+  if (!dims || (ndims != 1 && ndims != a->ndims_full)) return 1;
+  for (i = 0; i < a->ndims_full; i++) {
+    d[i] = (ndims == 1) ? dims[0] : dims[i];
+    if (d[i] <= 0) return 1;
+  }
+  return 0;
+}
+
+static void shapes(const app_def_t *a, const int64_t *d, int64_t rows[8], int64_t cols[8]) {
+  int i;
+  for (i = 0; i < 8; i++) { rows[i] = 1; cols[i] = 1; }
+  if (!strcmp(a->kind, "gemm")) {            /* NI, NJ, NK */
+    rows[0] = d[0]; cols[0] = d[2];          /* A NI x NK */
+    rows[1] = d[2]; cols[1] = d[1];          /* B NK x NJ */
+    rows[2] = d[0]; cols[2] = d[1];          /* C NI x NJ */
+  } else if (!strcmp(a->kind, "2mm")) {      /* NI, NJ, NK, NL */
+    rows[0] = d[0]; cols[0] = d[2];          /* A NI x NK */
+    rows[1] = d[2]; cols[1] = d[1];          /* B NK x NJ */
+    rows[2] = d[0]; cols[2] = d[1];          /* C NI x NJ */
+    rows[3] = d[1]; cols[3] = d[3];          /* D NJ x NL */
+    rows[4] = d[0]; cols[4] = d[3];          /* E NI x NL */
+  } else if (!strcmp(a->kind, "3mm")) {      /* NI, NJ, NK, NL, NM */
+    rows[0] = d[0]; cols[0] = d[2];          /* A NI x NK */
+    rows[1] = d[2]; cols[1] = d[1];          /* B NK x NJ */
+    rows[2] = d[1]; cols[2] = d[4];          /* C NJ x NM */
+    rows[3] = d[4]; cols[3] = d[3];          /* D NM x NL */
+    rows[4] = d[0]; cols[4] = d[1];          /* E NI x NJ */
+    rows[5] = d[1]; cols[5] = d[3];          /* F NJ x NL */
+    rows[6] = d[0]; cols[6] = d[3];          /* G NI x NL */
+  } else if (!strcmp(a->kind, "atax")) {     /* NX, NY */
+    rows[0] = d[0]; cols[0] = d[1];          /* A NX x NY */
+    cols[1] = d[1];                          /* x NY */
+    cols[2] = d[1];                          /* y NY */
+    cols[3] = d[0];                          /* tmp NX */
+  } else if (!strcmp(a->kind, "bicg")) {     /* NX, NY */
+    rows[0] = d[0]; cols[0] = d[1];          /* A NX x NY */
+    cols[1] = d[0];                          /* r NX */
+    cols[2] = d[1];                          /* s NY */
+    cols[3] = d[1];                          /* p NY */
+    cols[4] = d[0];                          /* q NX */
+  } else if (!strcmp(a->kind, "gesummv")) {  /* N */
+    rows[0] = d[0]; cols[0] = d[0];
+    rows[1] = d[0]; cols[1] = d[0];
+    cols[2] = d[0]; cols[3] = d[0]; cols[4] = d[0];
+  } else if (!strcmp(a->kind, "corr")) {     /* N rows, M cols */
+    rows[0] = d[0]; cols[0] = d[1];          /* data N x M */
+    cols[1] = d[1]; cols[2] = d[1];          /* mean, stddev M */
+    rows[3] = d[1]; cols[3] = d[1];          /* symmat M x M */
+  } else {                                   /* covar */
+    rows[0] = d[0]; cols[0] = d[1];
+    cols[1] = d[1];
+    rows[2] = d[1]; cols[2] = d[1];
+  }
+}
+
+int oracle_app_objects(const char *kind, const int64_t *dims, int ndims, oracle_object_info *info) {
+  const app_def_t *a = find_app(kind);
+  int64_t d[8], rows[8], cols[8];
+  int m;
+  if (!a || full_dims(a, dims, ndims, d)) return -1;
+  shapes(a, d, rows, cols);
+  if (info) {
+    for (m = 0; m < a->nobj; m++) {
+      info[m].name = a->names[m];
+      info[m].role = a->roles[m];
+      info[m].is_output = a->outputs[m];
+      info[m].rows = rows[m];
+      info[m].cols = cols[m];
+    }
+  }
+  return a->nobj;
+}
+
+/* default scalars (reading #18): gemm alpha,beta; gesummv alpha,beta; corr eps */
+static double scalar_or(const double *s, int i, double dflt) { return s ? s[i] : dflt; }
+
+static void app_gemm(obj_t *o, const int64_t *d, const double *sc) {
+  /* C <- alpha * (A . B) + beta * C   (R3 epilogue r = fma(alpha, acc, beta*C)) */
+  size_t NI = d[0], NJ = d[1], NK = d[2], i, j;
+  int T = W3(o[0].type, o[1].type, o[2].type);
+  double al = t_lit(T, scalar_or(sc, 0, 32412.0)), be = t_lit(T, scalar_or(sc, 1, 2123.0));
+  for (i = 0; i < NI; i++)
+    for (j = 0; j < NJ; j++) {
+      double acc = dot_chain(T, &o[0], i * NK, 1, &o[1], j, NJ, NK);
+      double bc = t_mul(T, be, ld(&o[2], i * NJ + j));
+      st(&o[2], i * NJ + j, t_fma(T, al, acc, bc), T);
+    }
+}
+
+/* out[i][j] <- sum_k A[i][k] B[k][j] (no epilogue), R3 order */
+static void matmul(obj_t *A, obj_t *B, obj_t *C, size_t NI, size_t NJ, size_t NK) {
+  size_t i, j;
+  int T = W3(A->type, B->type, C->type);
+  for (i = 0; i < NI; i++)
+    for (j = 0; j < NJ; j++) st(C, i * NJ + j, dot_chain(T, A, i * NK, 1, B, j, NJ, NK), T);
+}
+
+static void app_2mm(obj_t *o, const int64_t *d) {
+  size_t NI = d[0], NJ = d[1], NK = d[2], NL = d[3];
+  matmul(&o[0], &o[1], &o[2], NI, NJ, NK);   /* C <- A . B */
+  matmul(&o[2], &o[3], &o[4], NI, NL, NJ);   /* E <- C . D */
+}
+
+static void app_3mm(obj_t *o, const int64_t *d) {
+  size_t NI = d[0], NJ = d[1], NK = d[2], NL = d[3], NM = d[4];
+  matmul(&o[0], &o[1], &o[4], NI, NJ, NK);   /* E <- A . B */
+  matmul(&o[2], &o[3], &o[5], NJ, NL, NM);   /* F <- C . D */
+  matmul(&o[4], &o[5], &o[6], NI, NL, NJ);   /* G <- E . F */
+}
+
+static void app_atax(obj_t *o, const int64_t *d) {
+  size_t NX = d[0], NY = d[1], i, j;
+  int T1 = W3(o[0].type, o[1].type, o[3].type), T2 = W3(o[0].type, o[3].type, o[2].type);
+  for (i = 0; i < NX; i++) st(&o[3], i, rowdot(T1, &o[0], i * NY, NY, &o[1]), T1);  /* tmp <- A x */
+  for (j = 0; j < NY; j++) st(&o[2], j, colsum(T2, &o[0], NX, NY, j, &o[3], 0), T2); /* y <- A^T tmp */
+}
+
+static void app_bicg(obj_t *o, const int64_t *d) {
+  size_t NX = d[0], NY = d[1], i, j;
+  int T1 = W3(o[0].type, o[1].type, o[2].type), T2 = W3(o[0].type, o[3].type, o[4].type);
+  for (j = 0; j < NY; j++) st(&o[2], j, colsum(T1, &o[0], NX, NY, j, &o[1], 0), T1); /* s <- A^T r */
+  for (i = 0; i < NX; i++) st(&o[4], i, rowdot(T2, &o[0], i * NY, NY, &o[3]), T2);  /* q <- A p */
+}
+
+static void app_gesummv(obj_t *o, const int64_t *d, const double *sc) {
+  size_t N = d[0], i;
+  int T1 = W3(o[0].type, o[2].type, o[4].type);   /* tmp <- A x */
+  int T2 = W3(o[1].type, o[2].type, o[3].type);   /* y   <- B x */
+  int T3 = W2(o[4].type, o[3].type);              /* y   <- alpha tmp + beta y */
+  double al = t_lit(T3, scalar_or(sc, 0, 43532.0)), be = t_lit(T3, scalar_or(sc, 1, 12313.0));
+  for (i = 0; i < N; i++) st(&o[4], i, rowdot(T1, &o[0], i * N, N, &o[2]), T1);
+  for (i = 0; i < N; i++) st(&o[3], i, rowdot(T2, &o[1], i * N, N, &o[2]), T2);
+  for (i = 0; i < N; i++)
+    st(&o[3], i, t_fma(T3, al, ld(&o[4], i), t_mul(T3, be, ld(&o[3], i))), T3);
+}
+
+/* symmetric product sym[j1][j2] = sym[j2][j1] = sum_i X_ij1 X_ij2 (R3),
+ * j1 < j2 (diag_one) or j1 <= j2; divided by div if div != 0. */
+static void syrk_upper(obj_t *X, obj_t *S, size_t N, size_t M, int diag_one, double div_lit) {
+  size_t j1, j2;
+  int T = W2(X->type, S->type);
+  double dv = div_lit != 0.0 ? t_lit(T, div_lit) : 0.0;
+  for (j1 = 0; j1 < M; j1++) {
+    if (diag_one) st(S, j1 * M + j1, 1.0, T);
+    for (j2 = diag_one ? j1 + 1 : j1; j2 < M; j2++) {
+      double acc = dot_chain(T, X, j1, M, X, j2, M, N);
+      if (div_lit != 0.0) acc = t_div(T, acc, dv);
+      st(S, j1 * M + j2, acc, T);
+      st(S, j2 * M + j1, acc, T);
+    }
+  }
+}
+
+static void col_mean(obj_t *data, obj_t *mean, size_t N, size_t M) {
+  size_t j;
+  int T = W2(data->type, mean->type);
+  double n = t_lit(T, (double)N);
+  for (j = 0; j < M; j++) st(mean, j, t_div(T, colsum(T, data, N, M, j, NULL, 1), n), T);
+}
+
+static void app_corr(obj_t *o, const int64_t *d, const double *sc) {
+  size_t N = d[0], M = d[1], i, j;
+  int T2 = W3(o[0].type, o[1].type, o[2].type), T3 = T2;
+  double n2 = t_lit(T2, (double)N), eps = t_lit(T2, scalar_or(sc, 0, 0.005));
+  double sqn = t_lit(T3, sqrt((double)N));
+  col_mean(&o[0], &o[1], N, M);                                   /* mean */
+  for (j = 0; j < M; j++) {                                       /* stddev */
+    double s = t_sqrt(T2, t_div(T2, colsum(T2, &o[0], N, M, j, &o[1], 2), n2));
+    st(&o[2], j, s <= eps ? 1.0 : s, T2);
+  }
+  for (i = 0; i < N; i++)                                         /* normalise */
+    for (j = 0; j < M; j++) {
+      double dd = t_sub(T3, ld(&o[0], i * M + j), ld(&o[1], j));
+      st(&o[0], i * M + j, t_div(T3, dd, t_mul(T3, sqn, ld(&o[2], j))), T3);
+    }
+  syrk_upper(&o[0], &o[3], N, M, 1, 0.0);                         /* symmat */
+}
+
+static void app_covar(obj_t *o, const int64_t *d) {
+  size_t N = d[0], M = d[1], i, j;
+  int T2 = W2(o[0].type, o[1].type);
+  col_mean(&o[0], &o[1], N, M);                                   /* mean */
+  for (i = 0; i < N; i++)                                         /* centre */
+    for (j = 0; j < M; j++)
+      st(&o[0], i * M + j, t_sub(T2, ld(&o[0], i * M + j), ld(&o[1], j)), T2);
+  syrk_upper(&o[0], &o[2], N, M, 0, (double)N - 1.0);             /* symmat */
+}
+
+static int run_objects(const app_def_t *a, const int64_t *d, const double *sc, obj_t *o) {
+  if (!strcmp(a->kind, "gemm")) app_gemm(o, d, sc);
+  else if (!strcmp(a->kind, "2mm")) app_2mm(o, d);
+  else if (!strcmp(a->kind, "3mm")) app_3mm(o, d);
+  else if (!strcmp(a->kind, "atax")) app_atax(o, d);
+  else if (!strcmp(a->kind, "bicg")) app_bicg(o, d);
+  else if (!strcmp(a->kind, "gesummv")) app_gesummv(o, d, sc);
+  else if (!strcmp(a->kind, "corr")) app_corr(o, d, sc);
+  else app_covar(o, d);
+  return 0;
+}
+
+static void free_objects(obj_t *o, int n) {
+  int m;
+  for (m = 0; m < n; m++) free(o[m].p);
+}
+
+/* a2 + a3 */
+static int run_to_objects(const char *kind, const int64_t *dims, int ndims, const double *sc,
+                          const int *prec, const float *const *inputs, obj_t *o, const app_def_t **pa,
+                          int64_t *d) {
+  const app_def_t *a = find_app(kind);
+  int64_t rows[8], cols[8];
+  int m;
+  if (!a || full_dims(a, dims, ndims, d) || !prec) return 1;
+  shapes(a, d, rows, cols);
+  memset(o, 0, sizeof(obj_t) * 8);
+  for (m = 0; m < a->nobj; m++) {
+    if (prec[m] < 0 || prec[m] > 2) { free_objects(o, m); return 1; }
+    o[m].type = prec[m];
+    o[m].n = (size_t)(rows[m] * cols[m]);
+    o[m].p = calloc(o[m].n ? o[m].n : 1, tsize(prec[m]));
+    if (!o[m].p) { free_objects(o, m); return 1; }
+    if (a->roles[m] == 0 || a->roles[m] == 2) {         /* a2: convert orig f32 -> c(m) */
+      if (!inputs || !inputs[m]) { free_objects(o, m + 1); return 1; }
+      oracle_convert(inputs[m], OR_F32, o[m].p, prec[m], o[m].n);
+    }
+  }
+  run_objects(a, d, sc, o);
+  *pa = a;
+  return 0;
+}
+
+int oracle_run_config(const char *kind, const int64_t *dims, int ndims, const double *sc,
+                      const int *prec, const float *const *inputs, void *const *finals) {
+  obj_t o[8];
+  const app_def_t *a;
+  int64_t d[8];
+  int m;
+  if (run_to_objects(kind, dims, ndims, sc, prec, inputs, o, &a, d)) return 1;
+  for (m = 0; m < a->nobj; m++)
+    if (finals && finals[m]) memcpy(finals[m], o[m].p, o[m].n * tsize(o[m].type));
+  free_objects(o, a->nobj);
+  return 0;
+}
+
+int oracle_evaluate(const char *kind, const int64_t *dims, int ndims, const double *sc,
+                    const int *prec, const float *const *inputs, const double *const *ref,
+                    float *const *delivered, oracle_quality_result *res) {
+  obj_t o[8];
+  const app_def_t *a;
+  int64_t d[8];
+  int m;
+  double s = 0.0, mx = 0.0;
+  uint64_t nf = 0, n = 0;
+  if (!ref || !res) return 1;
+  if (run_to_objects(kind, dims, ndims, sc, prec, inputs, o, &a, d)) return 1;
+  for (m = 0; m < a->nobj; m++) {
+    float *buf;
+    if (!a->outputs[m]) continue;
+    /* a4: back-conversion c(o) -> orig (f32) */
+    buf = (delivered && delivered[m]) ? delivered[m] : (float *)malloc(o[m].n * 4 + 4);
+    oracle_convert(o[m].p, o[m].type, buf, OR_F32, o[m].n);
+    /* a5: quality of the delivered output vs the fp64 run */
+    oracle_quality_accumulate(buf, OR_F32, ref[m], o[m].n, &s, &mx, &nf);
+    n += o[m].n;
+    if (!(delivered && delivered[m])) free(buf);
+  }
+  free_objects(o, a->nobj);
+  res->n = n;
+  res->mean_rel = n ? s / (double)n : 0.0;
+  res->quality = 1.0 - res->mean_rel;
+  res->max_rel = mx;
+  res->nonfinite = nf;
+  return 0;
+}
