@@ -1,0 +1,167 @@
+/*
+ * prescaler.h -- C ABI of libprescaler.so: the B200 (sm_100a) hot path of
+ * PreScaler (Kang, Choi, Park, CGO '20), i.e. the evaluation of ONE
+ * memory-object-level mixed-precision configuration:
+ *
+ *   RunApp(config) -> KernelTime, TransferTime, Accuracy   (Alg. 1 line 8)
+ *   if Accuracy < TOQ then fail                            (Alg. 1 line 10)
+ *
+ * ("P:<n>" = line n of the paper text.)  Every floating-point rule not fixed by
+ * the paper is a reading listed in DESIGN.md §3 (R1-R6).
+ *
+ * Conventions
+ *  - Device pointers are CALLER-OWNED (e.g. torch tensors); the library never
+ *    frees them.  Host pointers are read/written only during the call (or until
+ *    the stream is synchronised, where stated).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *  - Every call returns ps_status.  No C++ exception crosses the ABI.  Errors of
+ *    asynchronous work surface at the next synchronising call as PS_ERR_CUDA.
+ *    ps_last_error() returns a thread-local message for the last failure.
+ *  - Buffers of a dtype hold IEEE binary64 / binary32 / binary16 values.
+ *  - One ps_app per host thread / stream (not thread-safe per handle).
+ */
+#ifndef PRESCALER_H
+#define PRESCALER_H
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define PS_API __attribute__((visibility("default")))
+#else
+#define PS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* precision codes in the paper's descending-precision order */
+typedef enum { PS_F64 = 0, PS_F32 = 1, PS_F16 = 2 } ps_dtype;
+
+typedef enum {
+  PS_OK = 0,
+  PS_ERR_INVALID = 1,      /* null pointer, bad dtype, id >= 3^M, wrong ndims, overlap */
+  PS_ERR_UNSUPPORTED = 2,  /* unknown app kind / dims out of range                    */
+  PS_ERR_CUDA = 3,         /* CUDA runtime error (message in ps_last_error())          */
+  PS_ERR_WORKSPACE = 4     /* workspace missing or smaller than ps_app_workspace_bytes */
+} ps_status;
+
+typedef enum {
+  PS_METRIC_MRE = 0,       /* quality = 1 - mean capped relative error        */
+  PS_METRIC_MAX_REL = 1    /* quality = 1 - min(1, max uncapped relative error)       */
+} ps_metric;
+
+PS_API const char *ps_status_string(int status);
+PS_API const char *ps_last_error(void);
+PS_API const char *ps_version(void);
+
+/* ------------------------------------------------------------------------- */
+/* (1) Device-side type conversion of one memory object (Fig. 3c). */
+/*   dst[i] = RNE_{dst_type}(src[i]) for i < n; widening is exact; subnormals   */
+/*   kept; overflow -> +-inf; NaN -> canonical NaN (f16 0x7FFF, f32 0x7FFFFFFF, */
+/*   f64 0x7FFFFFFFFFFFFFFF).  f64 -> f16 is a single rounding.  src, dst: device */
+/*   pointers, any alignment (16-byte aligned pointers take the vector path);    */
+/*   overlapping ranges -> PS_ERR_INVALID; n == 0 is a no-op; src_type ==        */
+/*   dst_type is a device-to-device copy.  Asynchronous on `stream`.             */
+PS_API ps_status ps_convert(const void *src, int src_type, void *dst, int dst_type, size_t n,
+                     void *stream);
+
+/* ------------------------------------------------------------------------- */
+/* (2) Output quality of one buffer against the fp64 run (reading #7):   */
+/*   e_i = 0 if o == r; 1 if o or r non-finite or r == 0; else                  */
+/*   min(1, |o - r| / |r|), with o = out[i] widened exactly to fp64.           */
+/*   res: mean_rel = sum(e)/n, max_rel = max uncapped relative error (inf on    */
+/*   overflow), nonfinite = #non-finite o, quality per `metric`.  out (out_type)*/
+/*   and ref (fp64): device pointers of n elements.  Synchronises `stream` and  */
+/*   writes the host struct *res.  Uses a small library-owned device scratch.   */
+typedef struct {
+  double quality, mean_rel, max_rel;
+  uint64_t n, nonfinite;
+} ps_quality_result;
+PS_API ps_status ps_quality(const void *out, int out_type, const double *ref, size_t n, int metric,
+                     void *stream, ps_quality_result *res);
+
+/* ------------------------------------------------------------------------- */
+/* (3) Applications: memory objects + statements (SURVEY c-4).   */
+/*   kind:  "gemm" dims {NI,NJ,NK}    scalars {alpha,beta} (default 32412,2123) */
+/*          "2mm"  dims {NI,NJ,NK,NL}                                          */
+/*          "3mm"  dims {NI,NJ,NK,NL,NM}                                       */
+/*          "atax" dims {NX,NY}   "bicg" dims {NX,NY}                          */
+/*          "gesummv" dims {N}    scalars {alpha,beta} (default 43532,12313)    */
+/*          "corr" dims {N,M} scalars {eps} (default 0.005)  "covar" dims {N,M} */
+/*   ndims == 1 sets every dimension to dims[0].  scalars may be NULL.          */
+/*   Every object's original precision is f32 (BASELINE).  Object order is the  */
+/*   configuration-id digit order.                                              */
+typedef struct ps_app ps_app;
+typedef struct {
+  const char *name;   /* static string owned by the library */
+  uint64_t n;         /* elements = rows * cols */
+  int64_t rows, cols; /* row-major */
+  int32_t orig;       /* ps_dtype of the original program (PS_F32) */
+  int32_t role;       /* 0 in, 1 out, 2 inout, 3 temp */
+  int32_t is_output;  /* delivered to the host and scored (a4/a5) */
+  int32_t reserved;
+} ps_object_info;
+
+PS_API ps_status ps_app_create(const char *kind, const int64_t *dims, int ndims, const double *scalars,
+                        ps_app **out);
+PS_API ps_status ps_app_destroy(ps_app *app);
+PS_API int ps_app_num_objects(const ps_app *app);            /* -1 if app == NULL */
+PS_API ps_status ps_app_object_info(const ps_app *app, int m, ps_object_info *out);
+/* flags: PS_FLAG_NO_TENSOR_CORES forces the SIMT contraction path for fp16   */
+/* operands (bit-exact with R3) instead of tcgen05 (tolerance R6).            */
+#define PS_FLAG_NO_TENSOR_CORES 1u
+PS_API ps_status ps_app_set_flags(ps_app *app, uint32_t flags);
+/* Device workspace the caller must allocate (>= 256-byte aligned). */
+PS_API size_t ps_app_workspace_bytes(const ps_app *app);
+/* Bind the workspace and the caller's device buffers:
+ *   orig_inputs[m]:  f32 device buffer (n elements) for role in/inout, else NULL;
+ *                    never modified (inout objects are copied into the workspace);
+ *   orig_outputs[m]: f32 device buffer receiving the back-converted output of every
+ *                    is_output object (a4), else NULL. */
+PS_API ps_status ps_app_bind(ps_app *app, void *workspace, size_t bytes, void *const *orig_inputs,
+                      void *const *orig_outputs);
+/* Copy host (preferably pinned) f32 inputs into the bound orig_inputs (H2D). */
+PS_API ps_status ps_app_load_host(ps_app *app, const void *const *host_inputs, void *stream);
+/* a0: run the all-f64 configuration (id 0) and copy the raw fp64 contents of each
+ * output object into ref_outputs[m] (caller-owned device, n elements; NULL for
+ * non-outputs).  These buffers become the quality reference of later calls. */
+PS_API ps_status ps_app_reference(ps_app *app, double *const *ref_outputs, void *stream);
+/* Use externally computed fp64 reference outputs instead (e.g. gathered). */
+PS_API ps_status ps_app_set_reference(ps_app *app, const double *const *ref_outputs);
+
+/* ------------------------------------------------------------------------- */
+/* (4) Evaluate one configuration (the hot path).                              */
+typedef struct {
+  uint64_t config_id;
+  float convert_ms;   /* a2: input conversion (incl. inout copies)            */
+  float kernel_ms;    /* a3: precision-scaled kernels                          */
+  float backconv_ms;  /* a4+a5 fused: back-conversion + per-element error      */
+  float quality_ms;   /* a5: final deterministic reduction                     */
+  float total_ms;     /* convert + kernel + backconv  (reading #19)            */
+  float reserved;
+  double quality;     /* 1 - mean relative error                               */
+  double max_rel;     /* max uncapped relative error                           */
+  uint64_t nonfinite; /* non-finite delivered output elements                  */
+  int32_t pass;       /* quality >= toq                                        */
+  int32_t status;     /* ps_status of this evaluation                          */
+} ps_result;          /* 64 bytes */
+
+/* id = sum_m code(prec[m]) * 3^m  (object 0 least significant) */
+PS_API ps_status ps_config_encode(const ps_app *app, const int *prec, uint64_t *id);
+PS_API ps_status ps_config_decode(const ps_app *app, uint64_t id, int *prec);
+/* prec: num_objects ps_dtype codes.  out == NULL: enqueue only (no sync, no record).
+ * Requires ps_app_bind and a reference (ps_app_reference / ps_app_set_reference). */
+PS_API ps_status ps_run_config(ps_app *app, const int *prec, double toq, void *stream, ps_result *out);
+
+/* ------------------------------------------------------------------------- */
+/* (5) Evaluate a list of configuration ids (a7).  results[i] for config_ids[i] */
+/* (host array).  *best_index = index of the fastest passing config (ties ->   */
+/* lowest id), -1 if none passes.  One stream synchronisation at the end.      */
+PS_API ps_status ps_sweep(ps_app *app, const uint64_t *config_ids, size_t n_configs, double toq,
+                   void *stream, ps_result *results, int64_t *best_index);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PRESCALER_H */

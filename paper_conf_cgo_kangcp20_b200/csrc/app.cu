@@ -1,0 +1,599 @@
+// app.cu -- ps_app: memory objects + statements of the PolyBench-shaped apps,
+// the configuration codec (a1), one-configuration evaluation ps_run_config
+// (a2-a6) and the sweep ps_sweep (a7).
+//
+// Evaluation of one configuration on one stream, no host synchronisation:
+//   ev0 | a2: each object read before written is converted orig(f32) -> c(m)
+//       |     into its workspace slot (c(m) == f32 inputs are used in place)
+//   ev1 | a3: statements in order; each picks its kernel from its compute type
+//       |     T = W(objects touched, f32) (R2): tcgen05 for fp16 x fp16 -> f32
+//       |     contractions, SIMT FFMA/DFMA otherwise, warp-shuffle mat-vec
+//   ev2 | a4+a5: per output object one fused back-convert + error kernel
+//   ev3 | a5: deterministic final reduction into this config's result slot
+//   ev4
+// A sweep enqueues a batch of configurations back to back and synchronises
+// once; the host then turns the (sum e, max, count) triples into ps_result.
+#include <math.h>
+#include <stdarg.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "common.cuh"
+#include "kernels.cuh"
+
+namespace ps {
+
+// ------------------------------------------------------------- errors
+static thread_local char g_err[512] = "";
+void set_error(const char *fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+}
+ps_status cuda_status(cudaError_t e, const char *what) {
+  set_error("CUDA error %d (%s) in %s", (int)e, cudaGetErrorString(e), what);
+  return PS_ERR_CUDA;
+}
+int num_sms() {
+  static int cached[64] = {0};
+  int d = 0;
+  cudaGetDevice(&d);
+  if (d < 0 || d >= 64) return 148;
+  if (!cached[d]) {
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d);
+    cached[d] = v > 0 ? v : 148;
+  }
+  return cached[d];
+}
+
+// ----------------------------------------------------------- app tables
+struct ObjDef {
+  const char *name;
+  int role;       // 0 in, 1 out, 2 inout, 3 temp
+  int is_output;  // delivered + scored
+};
+struct AppDef {
+  const char *kind;
+  int nobj;
+  int ndims;
+  ObjDef o[8];
+};
+// object order = configuration digit order
+static const AppDef kApps[] = {
+    {"gemm", 3, 3, {{"A", 0, 0}, {"B", 0, 0}, {"C", 2, 1}}},
+    {"2mm", 5, 4, {{"A", 0, 0}, {"B", 0, 0}, {"C", 3, 0}, {"D", 0, 0}, {"E", 1, 1}}},
+    {"3mm", 7, 5,
+     {{"A", 0, 0}, {"B", 0, 0}, {"C", 0, 0}, {"D", 0, 0}, {"E", 3, 0}, {"F", 3, 0}, {"G", 1, 1}}},
+    {"atax", 4, 2, {{"A", 0, 0}, {"x", 0, 0}, {"y", 1, 1}, {"tmp", 3, 0}}},
+    {"bicg", 5, 2, {{"A", 0, 0}, {"r", 0, 0}, {"s", 1, 1}, {"p", 0, 0}, {"q", 1, 1}}},
+    {"gesummv", 5, 1, {{"A", 0, 0}, {"B", 0, 0}, {"x", 0, 0}, {"y", 1, 1}, {"tmp", 3, 0}}},
+    {"corr", 4, 2, {{"data", 2, 0}, {"mean", 3, 0}, {"stddev", 3, 0}, {"symmat", 1, 1}}},
+    {"covar", 3, 2, {{"data", 2, 0}, {"mean", 3, 0}, {"symmat", 1, 1}}},
+};
+enum AppKind { K_GEMM, K_2MM, K_3MM, K_ATAX, K_BICG, K_GESUMMV, K_CORR, K_COVAR };
+
+}  // namespace ps
+
+using namespace ps;
+
+static constexpr int MAX_BATCH = 4096;
+static constexpr int NEV = 5;
+
+struct ps_app {
+  const AppDef *def = nullptr;
+  int kind = 0;
+  int64_t d[5] = {0, 0, 0, 0, 0};
+  int64_t rows[8] = {0}, cols[8] = {0};
+  double sc[2] = {0, 0};
+  uint32_t flags = 0;
+  // binding
+  char *ws = nullptr;
+  size_t ws_bytes = 0;
+  const float *orig_in[8] = {nullptr};
+  float *orig_out[8] = {nullptr};
+  const double *ref[8] = {nullptr};
+  bool bound = false, has_ref = false;
+  // workspace layout
+  size_t slot_off[8] = {0};
+  size_t partial_off = 0, qparts_off = 0, qres_off = 0, total = 0;
+  // timing
+  std::vector<cudaEvent_t> ev;
+  QPart *host_res = nullptr;   // pinned, MAX_BATCH
+  int device = -1;
+  ~ps_app() {
+    for (auto e : ev) cudaEventDestroy(e);
+    if (host_res) cudaFreeHost(host_res);
+  }
+};
+
+namespace {
+
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+void shapes(ps_app *a) {
+  const int64_t *d = a->d;
+  for (int m = 0; m < 8; m++) a->rows[m] = a->cols[m] = 1;
+  auto set = [&](int m, int64_t r, int64_t c) { a->rows[m] = r; a->cols[m] = c; };
+  switch (a->kind) {
+    case K_GEMM: set(0, d[0], d[2]); set(1, d[2], d[1]); set(2, d[0], d[1]); break;
+    case K_2MM:
+      set(0, d[0], d[2]); set(1, d[2], d[1]); set(2, d[0], d[1]); set(3, d[1], d[3]);
+      set(4, d[0], d[3]);
+      break;
+    case K_3MM:
+      set(0, d[0], d[2]); set(1, d[2], d[1]); set(2, d[1], d[4]); set(3, d[4], d[3]);
+      set(4, d[0], d[1]); set(5, d[1], d[3]); set(6, d[0], d[3]);
+      break;
+    case K_ATAX: set(0, d[0], d[1]); set(1, 1, d[1]); set(2, 1, d[1]); set(3, 1, d[0]); break;
+    case K_BICG:
+      set(0, d[0], d[1]); set(1, 1, d[0]); set(2, 1, d[1]); set(3, 1, d[1]); set(4, 1, d[0]);
+      break;
+    case K_GESUMMV:
+      set(0, d[0], d[0]); set(1, d[0], d[0]); set(2, 1, d[0]); set(3, 1, d[0]); set(4, 1, d[0]);
+      break;
+    case K_CORR: set(0, d[0], d[1]); set(1, 1, d[1]); set(2, 1, d[1]); set(3, d[1], d[1]); break;
+    case K_COVAR: set(0, d[0], d[1]); set(1, 1, d[1]); set(2, d[1], d[1]); break;
+  }
+}
+
+size_t nelem(const ps_app *a, int m) { return (size_t)(a->rows[m] * a->cols[m]); }
+
+void layout(ps_app *a) {
+  size_t off = 0;
+  for (int m = 0; m < a->def->nobj; m++) {
+    a->slot_off[m] = off;
+    off = align_up(off + nelem(a, m) * 8, 256);
+  }
+  size_t pb = 0;
+  if (a->kind == K_ATAX || a->kind == K_BICG || a->kind == K_CORR || a->kind == K_COVAR)
+    pb = colsum_partial_bytes(a->d[0], a->d[1]);
+  a->partial_off = off;
+  off = align_up(off + pb, 256);
+  int nout = 0;
+  for (int m = 0; m < a->def->nobj; m++) nout += a->def->o[m].is_output;
+  a->qparts_off = off;
+  off = align_up(off + (size_t)nout * QBLOCKS_MAX * sizeof(QPart), 256);
+  a->qres_off = off;
+  off = align_up(off + (size_t)MAX_BATCH * sizeof(QPart), 256);
+  a->total = off;
+}
+
+// ----------------------------------------------------------- statements
+struct Ctx {
+  ps_app *a;
+  const int *prec;
+  void *ptr[8];
+  cudaStream_t st;
+};
+
+ps_status contraction(Ctx &c, GemmArgs g) {
+  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && g.A.type == PS_F16 &&
+                  g.B.type == PS_F16 && g.T == PS_F32 && gemm_tc_supported(g);
+  return tc ? gemm_tc_async(g, c.st) : gemm_simt_async(g, c.st);
+}
+
+// out(M x N, row-major) = X(M x K, row-major) . Y(K x N, row-major), R3
+ps_status matmul(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_t K) {
+  GemmArgs g{};
+  g.M = M; g.N = N; g.K = K;
+  g.A = MatDesc{c.ptr[x], c.prec[x], K, 1};
+  g.B = MatDesc{c.ptr[y], c.prec[y], N, 1};
+  g.C = c.ptr[out]; g.c_type = c.prec[out]; g.ldc = N;
+  g.epi = EPI_PLAIN;
+  g.T = compute_type({c.prec[x], c.prec[y], c.prec[out]});
+  return contraction(c, g);
+}
+
+// symmat(M x M) = data^T data over N rows, upper tiles + mirror (R3)
+ps_status syrk(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double div, int diag_one) {
+  GemmArgs g{};
+  g.M = M; g.N = M; g.K = N;
+  g.A = MatDesc{c.ptr[data], c.prec[data], 1, M};   // A(j1, i) = data[i][j1]
+  g.B = MatDesc{c.ptr[data], c.prec[data], M, 1};   // B(i, j2) = data[i][j2]
+  g.C = c.ptr[sym]; g.c_type = c.prec[sym]; g.ldc = M;
+  g.epi = epi; g.div = div;
+  g.upper_only = 1;
+  g.T = compute_type({c.prec[data], c.prec[sym]});
+  ps_status s = contraction(c, g);
+  if (s != PS_OK) return s;
+  return mirror_async(c.ptr[sym], c.prec[sym], M, diag_one, c.st);
+}
+
+ps_status run_statements(Ctx &c) {
+  ps_app *a = c.a;
+  const int64_t *d = a->d;
+  const int *p = c.prec;
+  void **P = c.ptr;
+  void *partial = a->ws + a->partial_off;
+  ps_status s = PS_OK;
+#define S_(x)                      \
+  do {                             \
+    if ((s = (x)) != PS_OK) return s; \
+  } while (0)
+  switch (a->kind) {
+    case K_GEMM: {   // C <- alpha (A.B) + beta C
+      GemmArgs g{};
+      g.M = d[0]; g.N = d[1]; g.K = d[2];
+      g.A = MatDesc{P[0], p[0], d[2], 1};
+      g.B = MatDesc{P[1], p[1], d[1], 1};
+      g.C = P[2]; g.c_type = p[2]; g.ldc = d[1];
+      g.Cin = P[2]; g.cin_type = p[2];
+      g.epi = EPI_AXPBY; g.alpha = a->sc[0]; g.beta = a->sc[1];
+      g.T = compute_type({p[0], p[1], p[2]});
+      S_(contraction(c, g));
+      break;
+    }
+    case K_2MM:
+      S_(matmul(c, 0, 1, 2, d[0], d[1], d[2]));   // C <- A.B
+      S_(matmul(c, 2, 3, 4, d[0], d[3], d[1]));   // E <- C.D
+      break;
+    case K_3MM:
+      S_(matmul(c, 0, 1, 4, d[0], d[1], d[2]));   // E <- A.B
+      S_(matmul(c, 2, 3, 5, d[1], d[3], d[4]));   // F <- C.D
+      S_(matmul(c, 4, 5, 6, d[0], d[3], d[1]));   // G <- E.F
+      break;
+    case K_ATAX:   // tmp <- A x ; y <- A^T tmp
+      S_(rowdot_async(P[0], p[0], d[1], P[1], p[1], P[3], p[3], d[0], d[1], c.st));
+      S_(colsum_async(P[0], p[0], d[1], P[3], p[3], P[2], p[2], d[0], d[1],
+                      compute_type({p[0], p[3], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st));
+      break;
+    case K_BICG:   // s <- A^T r ; q <- A p
+      S_(colsum_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], d[0], d[1],
+                      compute_type({p[0], p[1], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st));
+      S_(rowdot_async(P[0], p[0], d[1], P[3], p[3], P[4], p[4], d[0], d[1], c.st));
+      break;
+    case K_GESUMMV:   // tmp <- A x ; y <- B x ; y <- alpha tmp + beta y
+      S_(rowdot_async(P[0], p[0], d[0], P[2], p[2], P[4], p[4], d[0], d[0], c.st));
+      S_(rowdot_async(P[1], p[1], d[0], P[2], p[2], P[3], p[3], d[0], d[0], c.st));
+      S_(axpby_async(P[4], p[4], P[3], p[3], d[0], a->sc[0], a->sc[1], c.st));
+      break;
+    case K_CORR: {
+      const double n = (double)d[0];
+      S_(colsum_async(P[0], p[0], d[1], nullptr, PS_F32, P[1], p[1], d[0], d[1],
+                      compute_type({p[0], p[1]}), COL_SUM, FIN_MEAN, n, 0, partial, c.st));
+      S_(colsum_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], d[0], d[1],
+                      compute_type({p[0], p[1], p[2]}), COL_SQDEV, FIN_STDDEV, n, a->sc[0],
+                      partial, c.st));
+      S_(corr_normalize_async(P[0], p[0], P[1], p[1], P[2], p[2], d[0], d[1], sqrt(n), c.st));
+      S_(syrk(c, 0, 3, d[0], d[1], EPI_PLAIN, 0.0, 1));
+      break;
+    }
+    case K_COVAR: {
+      const double n = (double)d[0];
+      S_(colsum_async(P[0], p[0], d[1], nullptr, PS_F32, P[1], p[1], d[0], d[1],
+                      compute_type({p[0], p[1]}), COL_SUM, FIN_MEAN, n, 0, partial, c.st));
+      S_(covar_center_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st));
+      S_(syrk(c, 0, 2, d[0], d[1], EPI_DIV, n - 1.0, 0));
+      break;
+    }
+  }
+#undef S_
+  return PS_OK;
+}
+
+ps_status check_prec(const ps_app *a, const int *prec) {
+  if (!prec) { set_error("null precision vector"); return PS_ERR_INVALID; }
+  for (int m = 0; m < a->def->nobj; m++)
+    if (!dtype_ok(prec[m])) { set_error("bad precision code %d for object %d", prec[m], m); return PS_ERR_INVALID; }
+  return PS_OK;
+}
+
+ps_status ensure_events(ps_app *a, size_t n) {
+  int dev;
+  PS_CUDA(cudaGetDevice(&dev));
+  if (a->device != dev) {
+    for (auto e : a->ev) cudaEventDestroy(e);
+    a->ev.clear();
+    a->device = dev;
+  }
+  while (a->ev.size() < n) {
+    cudaEvent_t e;
+    PS_CUDA(cudaEventCreate(&e));
+    a->ev.push_back(e);
+  }
+  if (!a->host_res) PS_CUDA(cudaMallocHost(&a->host_res, sizeof(QPart) * MAX_BATCH));
+  return PS_OK;
+}
+
+// a2 .. a5 for one configuration; events ev[0..4] (nullptr = untimed)
+ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res,
+                         cudaEvent_t *ev, bool quality) {
+  Ctx c{a, prec, {nullptr}, st};
+  if (ev) PS_CUDA(cudaEventRecord(ev[0], st));
+  for (int m = 0; m < a->def->nobj; m++) {
+    c.ptr[m] = a->ws + a->slot_off[m];
+    const int role = a->def->o[m].role;
+    if (role == 0 || role == 2) {
+      if (role == 0 && prec[m] == PS_F32) {
+        c.ptr[m] = (void *)a->orig_in[m];   // original precision: used in place
+      } else {
+        ps_status s = convert_async(a->orig_in[m], PS_F32, c.ptr[m], prec[m], nelem(a, m), st);
+        if (s != PS_OK) return s;
+      }
+    }
+  }
+  if (ev) PS_CUDA(cudaEventRecord(ev[1], st));
+  ps_status s = run_statements(c);
+  if (s != PS_OK) return s;
+  if (ev) PS_CUDA(cudaEventRecord(ev[2], st));
+  if (!quality) return PS_OK;
+  QPart *parts = (QPart *)(a->ws + a->qparts_off);
+  int np = 0;
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!a->def->o[m].is_output) continue;
+    s = backconv_quality_async(c.ptr[m], prec[m], a->ref[m], a->orig_out[m], nelem(a, m),
+                               parts + np, st);
+    if (s != PS_OK) return s;
+    np += qblocks(nelem(a, m));
+  }
+  if (ev) PS_CUDA(cudaEventRecord(ev[3], st));
+  s = quality_finalize_async(parts, np, res, st);
+  if (s != PS_OK) return s;
+  if (ev) PS_CUDA(cudaEventRecord(ev[4], st));
+  return PS_OK;
+}
+
+uint64_t space(const ps_app *a) {
+  uint64_t s = 1;
+  for (int m = 0; m < a->def->nobj; m++) s *= 3;
+  return s;
+}
+
+void decode(const ps_app *a, uint64_t id, int *prec) {
+  for (int m = 0; m < a->def->nobj; m++) { prec[m] = (int)(id % 3); id /= 3; }
+}
+
+uint64_t n_outputs(const ps_app *a) {
+  uint64_t n = 0;
+  for (int m = 0; m < a->def->nobj; m++)
+    if (a->def->o[m].is_output) n += nelem(a, m);
+  return n;
+}
+
+float ms_between(cudaEvent_t x, cudaEvent_t y) {
+  float t = 0.f;
+  if (cudaEventElapsedTime(&t, x, y) != cudaSuccess) return NAN;
+  return t;
+}
+
+ps_status ready(const ps_app *a) {
+  if (!a) { set_error("null app"); return PS_ERR_INVALID; }
+  if (!a->bound) { set_error("app not bound (ps_app_bind)"); return PS_ERR_WORKSPACE; }
+  if (!a->has_ref) { set_error("no reference (ps_app_reference)"); return PS_ERR_INVALID; }
+  return PS_OK;
+}
+
+}  // namespace
+
+// ===================================================================== ABI
+extern "C" {
+
+const char *ps_status_string(int s) {
+  switch (s) {
+    case PS_OK: return "ok";
+    case PS_ERR_INVALID: return "invalid argument";
+    case PS_ERR_UNSUPPORTED: return "unsupported";
+    case PS_ERR_CUDA: return "cuda error";
+    case PS_ERR_WORKSPACE: return "workspace missing or too small";
+  }
+  return "unknown status";
+}
+const char *ps_last_error(void) { return g_err; }
+const char *ps_version(void) { return "prescaler-b200 0.1 (sm_100a)"; }
+
+ps_status ps_app_create(const char *kind, const int64_t *dims, int ndims, const double *scalars,
+                        ps_app **out) {
+  if (!kind || !dims || !out) { set_error("ps_app_create: null pointer"); return PS_ERR_INVALID; }
+  const AppDef *def = nullptr;
+  int k = 0;
+  for (size_t i = 0; i < sizeof(kApps) / sizeof(kApps[0]); i++)
+    if (!strcmp(kApps[i].kind, kind)) { def = &kApps[i]; k = (int)i; }
+  if (!def) { set_error("ps_app_create: unknown app '%s'", kind); return PS_ERR_UNSUPPORTED; }
+  if (ndims != 1 && ndims != def->ndims) {
+    set_error("ps_app_create: %s takes 1 or %d dims, got %d", kind, def->ndims, ndims);
+    return PS_ERR_INVALID;
+  }
+  ps_app *a = new ps_app();
+  a->def = def;
+  a->kind = k;
+  for (int i = 0; i < def->ndims; i++) {
+    a->d[i] = ndims == 1 ? dims[0] : dims[i];
+    if (a->d[i] <= 0 || a->d[i] > (int64_t)1 << 31) {
+      delete a;
+      set_error("ps_app_create: dimension out of range");
+      return PS_ERR_UNSUPPORTED;
+    }
+  }
+  if (k == K_GEMM) { a->sc[0] = 32412.0; a->sc[1] = 2123.0; }
+  if (k == K_GESUMMV) { a->sc[0] = 43532.0; a->sc[1] = 12313.0; }
+  if (k == K_CORR) { a->sc[0] = 0.005; }
+  if (scalars) {
+    if (k == K_GEMM || k == K_GESUMMV) { a->sc[0] = scalars[0]; a->sc[1] = scalars[1]; }
+    if (k == K_CORR) a->sc[0] = scalars[0];
+  }
+  shapes(a);
+  layout(a);
+  *out = a;
+  return PS_OK;
+}
+
+ps_status ps_app_destroy(ps_app *a) {
+  delete a;
+  return PS_OK;
+}
+
+int ps_app_num_objects(const ps_app *a) { return a ? a->def->nobj : -1; }
+
+ps_status ps_app_object_info(const ps_app *a, int m, ps_object_info *out) {
+  if (!a || !out || m < 0 || m >= a->def->nobj) { set_error("ps_app_object_info: bad argument"); return PS_ERR_INVALID; }
+  out->name = a->def->o[m].name;
+  out->rows = a->rows[m];
+  out->cols = a->cols[m];
+  out->n = (uint64_t)nelem(a, m);
+  out->orig = PS_F32;
+  out->role = a->def->o[m].role;
+  out->is_output = a->def->o[m].is_output;
+  out->reserved = 0;
+  return PS_OK;
+}
+
+ps_status ps_app_set_flags(ps_app *a, uint32_t flags) {
+  if (!a) { set_error("null app"); return PS_ERR_INVALID; }
+  a->flags = flags;
+  return PS_OK;
+}
+
+size_t ps_app_workspace_bytes(const ps_app *a) { return a ? a->total : 0; }
+
+ps_status ps_app_bind(ps_app *a, void *ws, size_t bytes, void *const *in, void *const *out) {
+  if (!a || !in || !out) { set_error("ps_app_bind: null pointer"); return PS_ERR_INVALID; }
+  if (!ws || bytes < a->total || ((uintptr_t)ws % 256)) {
+    set_error("ps_app_bind: workspace needs %zu bytes, 256-aligned", a->total);
+    return PS_ERR_WORKSPACE;
+  }
+  for (int m = 0; m < a->def->nobj; m++) {
+    const int role = a->def->o[m].role;
+    if ((role == 0 || role == 2) && !in[m]) { set_error("ps_app_bind: input %d missing", m); return PS_ERR_INVALID; }
+    if (a->def->o[m].is_output && !out[m]) { set_error("ps_app_bind: output %d missing", m); return PS_ERR_INVALID; }
+    a->orig_in[m] = (role == 0 || role == 2) ? (const float *)in[m] : nullptr;
+    a->orig_out[m] = a->def->o[m].is_output ? (float *)out[m] : nullptr;
+  }
+  a->ws = (char *)ws;
+  a->ws_bytes = bytes;
+  a->bound = true;
+  return PS_OK;
+}
+
+ps_status ps_app_load_host(ps_app *a, const void *const *host, void *stream) {
+  if (!a || !host) { set_error("ps_app_load_host: null pointer"); return PS_ERR_INVALID; }
+  if (!a->bound) { set_error("ps_app_load_host: app not bound"); return PS_ERR_WORKSPACE; }
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!a->orig_in[m]) continue;
+    if (!host[m]) { set_error("ps_app_load_host: host input %d missing", m); return PS_ERR_INVALID; }
+    PS_CUDA(cudaMemcpyAsync((void *)a->orig_in[m], host[m], nelem(a, m) * sizeof(float),
+                            cudaMemcpyHostToDevice, (cudaStream_t)stream));
+  }
+  return PS_OK;
+}
+
+ps_status ps_app_reference(ps_app *a, double *const *ref, void *stream) {
+  if (!a || !ref) { set_error("ps_app_reference: null pointer"); return PS_ERR_INVALID; }
+  if (!a->bound) { set_error("ps_app_reference: app not bound"); return PS_ERR_WORKSPACE; }
+  cudaStream_t st = (cudaStream_t)stream;
+  int prec[8] = {0};   // all f64 = configuration id 0
+  ps_status s = enqueue_config(a, prec, st, nullptr, nullptr, false);
+  if (s != PS_OK) return s;
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!a->def->o[m].is_output) continue;
+    if (!ref[m]) { set_error("ps_app_reference: ref %d missing", m); return PS_ERR_INVALID; }
+    PS_CUDA(cudaMemcpyAsync(ref[m], a->ws + a->slot_off[m], nelem(a, m) * 8,
+                            cudaMemcpyDeviceToDevice, st));
+    a->ref[m] = ref[m];
+  }
+  PS_CUDA(cudaStreamSynchronize(st));
+  a->has_ref = true;
+  return PS_OK;
+}
+
+ps_status ps_app_set_reference(ps_app *a, const double *const *ref) {
+  if (!a || !ref) { set_error("ps_app_set_reference: null pointer"); return PS_ERR_INVALID; }
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!a->def->o[m].is_output) continue;
+    if (!ref[m]) { set_error("ps_app_set_reference: ref %d missing", m); return PS_ERR_INVALID; }
+    a->ref[m] = ref[m];
+  }
+  a->has_ref = true;
+  return PS_OK;
+}
+
+ps_status ps_config_encode(const ps_app *a, const int *prec, uint64_t *id) {
+  if (!a || !id) { set_error("ps_config_encode: null pointer"); return PS_ERR_INVALID; }
+  ps_status s = check_prec(a, prec);
+  if (s != PS_OK) return s;
+  uint64_t v = 0, w = 1;
+  for (int m = 0; m < a->def->nobj; m++) { v += (uint64_t)prec[m] * w; w *= 3; }
+  *id = v;
+  return PS_OK;
+}
+
+ps_status ps_config_decode(const ps_app *a, uint64_t id, int *prec) {
+  if (!a || !prec) { set_error("ps_config_decode: null pointer"); return PS_ERR_INVALID; }
+  if (id >= space(a)) { set_error("ps_config_decode: id %llu >= 3^%d", (unsigned long long)id, a->def->nobj); return PS_ERR_INVALID; }
+  decode(a, id, prec);
+  return PS_OK;
+}
+
+static void fill_result(const ps_app *a, uint64_t id, const QPart &q, cudaEvent_t *ev, double toq,
+                        ps_result *r) {
+  const double n = (double)n_outputs(a);
+  memset(r, 0, sizeof(*r));
+  r->config_id = id;
+  r->convert_ms = ms_between(ev[0], ev[1]);
+  r->kernel_ms = ms_between(ev[1], ev[2]);
+  r->backconv_ms = ms_between(ev[2], ev[3]);
+  r->quality_ms = ms_between(ev[3], ev[4]);
+  r->total_ms = r->convert_ms + r->kernel_ms + r->backconv_ms;
+  r->quality = 1.0 - q.sum / n;
+  r->max_rel = q.mx;
+  r->nonfinite = q.nf;
+  r->pass = r->quality >= toq;   // Alg. 1 l.10: fail iff Accuracy < TOQ
+  r->status = PS_OK;
+}
+
+ps_status ps_run_config(ps_app *a, const int *prec, double toq, void *stream, ps_result *out) {
+  ps_status s = ready(a);
+  if (s != PS_OK) return s;
+  if ((s = check_prec(a, prec)) != PS_OK) return s;
+  if ((s = ensure_events(a, NEV)) != PS_OK) return s;
+  cudaStream_t st = (cudaStream_t)stream;
+  QPart *res = (QPart *)(a->ws + a->qres_off);
+  s = enqueue_config(a, prec, st, res, out ? a->ev.data() : nullptr, true);
+  if (s != PS_OK) return s;
+  if (!out) return PS_OK;
+  PS_CUDA(cudaMemcpyAsync(a->host_res, res, sizeof(QPart), cudaMemcpyDeviceToHost, st));
+  PS_CUDA(cudaStreamSynchronize(st));
+  uint64_t id = 0;
+  ps_config_encode(a, prec, &id);
+  fill_result(a, id, a->host_res[0], a->ev.data(), toq, out);
+  return PS_OK;
+}
+
+ps_status ps_sweep(ps_app *a, const uint64_t *ids, size_t n, double toq, void *stream,
+                   ps_result *results, int64_t *best) {
+  ps_status s = ready(a);
+  if (s != PS_OK) return s;
+  if ((n && (!ids || !results)) || !best) { set_error("ps_sweep: null pointer"); return PS_ERR_INVALID; }
+  const uint64_t sp = space(a);
+  for (size_t i = 0; i < n; i++)
+    if (ids[i] >= sp) { set_error("ps_sweep: config id %llu out of range", (unsigned long long)ids[i]); return PS_ERR_INVALID; }
+  cudaStream_t st = (cudaStream_t)stream;
+  QPart *res = (QPart *)(a->ws + a->qres_off);
+  *best = -1;
+  for (size_t b0 = 0; b0 < n; b0 += MAX_BATCH) {
+    const size_t nb = std::min((size_t)MAX_BATCH, n - b0);
+    if ((s = ensure_events(a, nb * NEV)) != PS_OK) return s;
+    for (size_t i = 0; i < nb; i++) {
+      int prec[8];
+      decode(a, ids[b0 + i], prec);
+      s = enqueue_config(a, prec, st, res + i, a->ev.data() + i * NEV, true);
+      if (s != PS_OK) return s;
+    }
+    PS_CUDA(cudaMemcpyAsync(a->host_res, res, sizeof(QPart) * nb, cudaMemcpyDeviceToHost, st));
+    PS_CUDA(cudaStreamSynchronize(st));
+    for (size_t i = 0; i < nb; i++)
+      fill_result(a, ids[b0 + i], a->host_res[i], a->ev.data() + i * NEV, toq, &results[b0 + i]);
+  }
+  for (size_t i = 0; i < n; i++) {
+    if (!results[i].pass) continue;
+    if (*best < 0 || results[i].total_ms < results[*best].total_ms ||
+        (results[i].total_ms == results[*best].total_ms && results[i].config_id < results[*best].config_id))
+      *best = (int64_t)i;
+  }
+  return PS_OK;
+}
+
+}  // extern "C"

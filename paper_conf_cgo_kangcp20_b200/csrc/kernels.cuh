@@ -1,0 +1,78 @@
+// kernels.cuh -- internal launcher declarations of libprescaler (not part of the ABI).
+#pragma once
+#include "common.cuh"
+
+namespace ps {
+
+// ------------------------------------------------------------ conversion (a2)
+ps_status convert_async(const void *src, int st, void *dst, int dt, size_t n, cudaStream_t stream);
+
+// ------------------------------------------------------- quality (a4 + a5)
+constexpr int QTHREADS = 256;
+constexpr int QBLOCKS_MAX = 1024;   // fixed, SM-count independent (determinism)
+struct QPart {
+  double sum;
+  double mx;
+  unsigned long long nf;
+};
+int qblocks(size_t n);
+// delivered == nullptr: score the exact widened value, no write (ps_quality)
+ps_status backconv_quality_async(const void *out, int out_type, const double *ref, float *delivered,
+                                 size_t n, QPart *parts, cudaStream_t st);
+ps_status quality_finalize_async(const QPart *parts, int nparts, QPart *res, cudaStream_t st);
+
+// ------------------------------------------------------ contractions (a3)
+// element (r, c) of a matrix operand lives at p[r * s_row + c * s_col]
+struct MatDesc {
+  const void *p;
+  int type;
+  int64_t s_row, s_col;
+};
+enum Epilogue { EPI_PLAIN = 0, EPI_AXPBY = 1 /* fma(alpha, acc, beta*Cin) */, EPI_DIV = 2 };
+struct GemmArgs {
+  int64_t M, N, K;
+  MatDesc A;            // A(i, k), M x K
+  MatDesc B;            // B(k, j), K x N
+  void *C;              // output, row-major, leading dimension ldc
+  int c_type;
+  int64_t ldc;
+  const void *Cin;      // EPI_AXPBY: previous contents of C (row-major, ldc)
+  int cin_type;
+  int epi;
+  double alpha, beta, div;   // fp64 literals (rounded to T on the device side)
+  int upper_only;       // SYRK: skip tiles strictly below the diagonal
+  int T;                // compute type PS_F32 / PS_F64
+};
+// R3-exact SIMT contraction (FFMA / DFMA fma chains, k ascending)
+ps_status gemm_simt_async(const GemmArgs &g, cudaStream_t st);
+// tcgen05 tensor-core contraction for fp16 x fp16 -> f32 accumulate (R6)
+bool gemm_tc_supported(const GemmArgs &g);
+ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st);
+// S[j1][j2] := S[j2][j1] for j1 > j2; diag := 1 if diag_one (SYRK mirror)
+ps_status mirror_async(void *S, int type, int64_t M, int diag_one, cudaStream_t st);
+
+// ------------------------------------------------------------ mat-vec (a3)
+constexpr int ROWDOT_LANES = 32;     // R5
+constexpr int COLSUM_CHUNK = 256;    // R5
+// out[i] = RNE_out( butterfly( lane fma chains ) ), R5 row-dot
+ps_status rowdot_async(const void *A, int ta, int64_t lda, const void *x, int tx, void *out,
+                       int tout, int64_t rows, int64_t cols, cudaStream_t st);
+// column sums over 256-row chunks:
+//   mode 0: p = fma(A_ij, w_i, p)   mode 1: p = p + A_ij   mode 2: d = A_ij - w_j, p = fma(d, d, p)
+// finalize: 0 plain, 1 total / n, 2 stddev (sqrt(total / n), <= eps -> 1)
+enum ColMode { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
+enum ColFin { FIN_PLAIN = 0, FIN_MEAN = 1, FIN_STDDEV = 2 };
+size_t colsum_partial_bytes(int64_t rows, int64_t cols);
+ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
+                       int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
+                       double eps, void *partial, cudaStream_t st);
+// y_i = RNE_y(fma(alpha, tmp_i, beta * y_i)) in T = W(tmp, y)
+ps_status axpby_async(const void *tmp, int ttmp, void *y, int ty, int64_t n, double alpha,
+                      double beta, cudaStream_t st);
+// CORR: data_ij = (data_ij - mean_j) / (sqrt_n * std_j)   COVAR: data_ij -= mean_j
+ps_status corr_normalize_async(void *data, int td, const void *mean, int tm, const void *std,
+                               int ts, int64_t rows, int64_t cols, double sqrt_n, cudaStream_t st);
+ps_status covar_center_async(void *data, int td, const void *mean, int tm, int64_t rows,
+                             int64_t cols, cudaStream_t st);
+
+}  // namespace ps
