@@ -1,0 +1,482 @@
+#!/usr/bin/env python
+"""bench.py -- PreScaler configuration-evaluation throughput on B200.
+
+A "step" is one pass of the whole hot path over the
+workload: for every app, the fp64 reference run (a0) and the evaluation of its
+full configuration space 3^M (a1 decode, a2 conversion, a3 precision-scaled
+kernels, a4+a5 fused back-conversion + quality, a6 records, a7 best config).
+Default workload = BASELINE.json configs[2]: ATAX, BICG, GESUMMV at N=16384
+(81 + 243 + 243 = 567 configurations per step), Table 4 "Default" inputs,
+TOQ 0.9.  configs[1] (the conversion sweep) is a single row (a2) of the path,
+so it is reported as the secondary `conversion_gbs` key, not as the step.
+
+Multi-GPU (torchrun, one process per GPU): the config space of every app is
+partitioned across ranks (deterministic LPT over a cost model); each rank
+evaluates its share; one NCCL all_gather of the 64-byte result records per app
+per step.  Timing: barrier + synchronize on both sides of exactly --steps
+steps, CUDA events on the launching stream, max over ranks.
+
+--impl reference times the CPU oracle (oracle/, the plain C definition) as it
+stands on the host cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # BASELINE.json configs[2] (default)
+    "matvec": [("atax", [16384, 16384]), ("bicg", [16384, 16384]), ("gesummv", [16384])],
+    # BASELINE.json configs[0]
+    "gemm64": [("gemm", [64])],
+    # BASELINE.json configs[3] / configs[4]
+    "contract": [("2mm", [8192]), ("3mm", [8192])],
+    "corr": [("corr", [8192, 8192]), ("covar", [8192, 8192])],
+}
+SIZE = {0: 8, 1: 4, 2: 2}
+# CPU-oracle samples: (reduced dimension, work exponent) -- the oracle needs ~40 s
+# per ATAX configuration at N=16384, so the CPU legs run every app dimension at
+# the reduced size and extrapolate throughput by (N_sample / N)^exponent (O(N^2)
+# mat-vec, O(N^3) contractions); labelled "extrapolated" in the JSON.
+CPU_SAMPLE = {"matvec": (8192, 2), "gemm64": (None, 0), "contract": (384, 3), "corr": (512, 3)}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), float(p["bf16_tflops"]), "measured"
+    except Exception:
+        return 6650.0, 1590.0, "fallback"
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index, self.proc = index, None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out, _ = self.proc.communicate()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": float(max(mx)) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------- algorithmic bytes
+def kernel_bytes(kind, dims, prec):
+    """Algorithmic bytes of the a3 statement kernels of one configuration (one
+    streaming pass over each matrix) + the vectors."""
+    n = dims[0]
+    if kind == "atax":
+        return n * n * SIZE[prec[0]] + n * (SIZE[prec[1]] + SIZE[prec[2]] + 2 * SIZE[prec[3]])
+    if kind == "bicg":
+        return n * n * SIZE[prec[0]] + n * sum(SIZE[prec[k]] for k in (1, 2, 3, 4))
+    if kind == "gesummv":
+        return n * n * (SIZE[prec[0]] + SIZE[prec[1]]) + n * (SIZE[prec[2]] + 3 * SIZE[prec[3]] +
+                                                            2 * SIZE[prec[4]])
+    return None
+
+
+def convert_bytes(objects, prec):
+    b = 0
+    for o, p in zip(objects, prec):
+        if o["role"] in (0, 2) and (p != 1 or o["role"] == 2):
+            b += o["n"] * (4 + SIZE[p])
+    return b
+
+
+def decode(cid, m):
+    out = []
+    for _ in range(m):
+        out.append(cid % 3)
+        cid //= 3
+    return out
+
+
+# ---------------------------------------------------------- reference arm
+def _sample(workload):
+    kind, dims = WORKLOADS[workload][0]
+    n_s, expo = CPU_SAMPLE[workload]
+    sdims = dims if n_s is None else [n_s] * len(dims)
+    factor = 1.0 if n_s is None else (n_s / float(dims[0])) ** expo
+    return kind, dims, sdims, factor, expo
+
+
+def run_reference_arm(args, rank, world):
+    """The CPU oracle as it stands (single-threaded), bounded sample per step."""
+    import oracle
+    from paper_conf_cgo_kangcp20_b200 import inputs as gen
+    if rank != 0:
+        return 0
+    kind, dims, sdims, factor, expo = _sample(args.workload)
+    objs = oracle.app_objects(kind, sdims)
+    ins = gen.make_inputs(kind, objs, args.input_set)
+    t0 = time.time()
+    ref = oracle.reference(kind, sdims, ins)
+    t_ref = time.time() - t0
+    m = len(objs)
+    cycle = [(3 ** m - 1) // 2, 3 ** m - 1, 0, 1]
+    for w in range(args.warmup):
+        oracle.evaluate(kind, sdims, decode(cycle[w % len(cycle)], m), ins, ref, toq=args.toq)
+    t0 = time.time()
+    for s in range(args.steps):
+        oracle.evaluate(kind, sdims, decode(cycle[s % len(cycle)], m), ins, ref, toq=args.toq)
+    el = time.time() - t0
+    v = args.steps / el * factor
+    sample = "%s %s: 1 configuration evaluation per step (ids cycling %s) at %s, fp64 " \
+             "reference precomputed (%.1f s); throughput extrapolated to %s by (N_s/N)^%d = %.4g" % (
+                 kind, "x".join(map(str, dims)), cycle, "x".join(map(str, sdims)), t_ref,
+                 "x".join(map(str, dims)), expo, factor)
+    line = {"impl": "reference", "metric": "configs evaluated/s", "value": v,
+            "unit": "configs/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": el / args.steps * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64/f32/f16 (per configuration)", "data": "synthetic",
+            "config": {"workload": args.workload, "sample": sample, "input_set": args.input_set,
+                       "toq": args.toq},
+            "cpu_baseline": {"value": v, "unit": "configs/s", "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": v, "unit": "configs/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline(args):
+    """Oracle timed on the host: the fp64 reference run (config 0) + the all-f32
+    configuration of the first app, at the sample size."""
+    import oracle
+    from paper_conf_cgo_kangcp20_b200 import inputs as gen
+    kind, dims, sdims, factor, expo = _sample(args.workload)
+    objs = oracle.app_objects(kind, sdims)
+    ins = gen.make_inputs(kind, objs, args.input_set)
+    m = len(objs)
+    ids = [(3 ** m - 1) // 2]
+    t0 = time.time()
+    ref = oracle.reference(kind, sdims, ins)
+    for cid in ids:
+        oracle.evaluate(kind, sdims, decode(cid, m), ins, ref, toq=args.toq)
+    el = time.time() - t0
+    n_eval = 1 + len(ids)
+    return {"value": n_eval / el * factor, "unit": "configs/s", "cores": 1, "kind": "oracle",
+            "sample": "%s at %s: fp64 reference run (config 0) + config %s (all-f32), single-"
+                      "threaded C oracle, %.1f s; extrapolated to %s by (N_s/N)^%d = %.4g" % (
+                          kind, "x".join(map(str, sdims)), ids, el, "x".join(map(str, dims)),
+                          expo, factor)}
+
+
+# ------------------------------------------------------------ conversion
+def conversion_sweep(torch, B, flush, reps=10):
+    out = {}
+    TD = {0: torch.float64, 1: torch.float32, 2: torch.float16}
+    for st, dt, name in [(1, 2, "f32->f16"), (2, 1, "f16->f32"), (0, 2, "f64->f16"),
+                         (0, 1, "f64->f32")]:
+        n = (1 << 30) // SIZE[st]           # 1 GiB source
+        src = torch.zeros(n, dtype=TD[st], device="cuda")
+        dst = torch.empty(n, dtype=TD[dt], device="cuda")
+        for _ in range(3):
+            B.ps_convert(src, st, dst, dt)
+        ts = []
+        for _ in range(reps):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            B.ps_convert(src, st, dst, dt)
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        t = float(np.median(ts))
+        out[name] = round(n * (SIZE[st] + SIZE[dt]) / (t * 1e-3) / 1e9, 1)
+        del src, dst
+    return out
+
+
+# ------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="matvec", choices=sorted(WORKLOADS))
+    ap.add_argument("--input-set", default="default", choices=["default", "random", "image"])
+    ap.add_argument("--toq", type=float, default=0.9)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-conversion", action="store_true")
+    ap.add_argument("--profile", action="store_true",
+                    help="one untimed-warmup-free step for ncu launch lists (not a bench number)")
+    args = ap.parse_args()
+    if args.profile:
+        args.warmup, args.steps = 0, 1
+        args.no_e2e = args.no_cpu_baseline = args.no_conversion = True
+    elif args.warmup < 3:
+        log("warmup raised to 3 (timing rule)")
+        args.warmup = 3
+
+    rank, world = int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.impl == "reference":
+        return run_reference_arm(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_cgo_kangcp20_b200 import binding as B
+    from paper_conf_cgo_kangcp20_b200 import build as build_mod
+    from paper_conf_cgo_kangcp20_b200 import dist as D
+    from paper_conf_cgo_kangcp20_b200 import inputs as gen
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if rank == 0:
+        build_mod.build()
+    if world > 1:
+        dist.barrier()
+    B.lib()
+    stream = torch.cuda.current_stream()
+
+    # ------------------------------------------------------------ setup (a0 inputs)
+    apps = []
+    for kind, dims in WORKLOADS[args.workload]:
+        app = B.App(kind, dims)
+        t0 = time.time()
+        ins = gen.make_inputs(kind, app.objects, args.input_set)
+        dins = [torch.from_numpy(a.reshape(-1)).cuda() if a is not None else None for a in ins]
+        app.bind(dins)
+        refs = app.reference()
+        ids = list(range(app.space))
+        mine = D.partition_configs(kind, dims, app.objects, ids, world, rank) if world > 1 else ids
+        apps.append(dict(kind=kind, dims=dims, app=app, ins=ins, refs=refs, ids=mine,
+                         space=app.space))
+        log("rank %d setup %s %s: %d/%d configs, %.1f s" % (rank, kind, dims, len(mine),
+                                                              app.space, time.time() - t0))
+    total_configs = sum(a["space"] for a in apps)
+
+    def step(collect=None):
+        for a in apps:
+            a["app"].reference(refs=a["refs"])                       # a0
+            arr, _ = a["app"].sweep_raw(a["ids"], args.toq)          # a1-a7 (local share)
+            if world > 1:
+                arr = D.gather_results(arr)                          # NCCL gather
+            if collect is not None:
+                collect[a["kind"]] = arr
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # ----------------------------------------------------------------- timed
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    last = {}
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    l0 = B.ps_kernel_launches()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for s in range(args.steps):
+        step(last if s == args.steps - 1 else None)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = B.ps_kernel_launches() - l0
+    el_ms = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    if world > 1:
+        t = torch.tensor([el_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        el_ms = float(t.item())
+        lt = torch.tensor([launches], dtype=torch.int64, device="cuda")
+        dist.all_reduce(lt, op=dist.ReduceOp.SUM)
+        launches = int(lt.item())
+    value = total_configs * args.steps / (el_ms * 1e-3)
+
+    # ------------------------------------------------- e2e through host buffers
+    e2e = None
+    if not args.no_e2e:
+        host = []
+        h2d = 0
+        for a in apps:
+            hin = [torch.from_numpy(x.reshape(-1)).pin_memory() if x is not None else None
+                   for x in a["ins"]]
+            host.append(hin)
+            h2d += sum(x.numel() * 4 for x in hin if x is not None)
+        d2h = sum(len(a["ids"]) * 24 for a in apps)      # one (sum e, max, count) record per config
+
+        def step_e2e():
+            for a, hin in zip(apps, host):
+                a["app"].load_host(hin)                               # H2D of the inputs
+                a["app"].reference(refs=a["refs"])
+                arr, _ = a["app"].sweep_raw(a["ids"], args.toq)       # results read back (D2H)
+                if world > 1:
+                    D.gather_results(arr)
+        step_e2e()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.steps):
+            step_e2e()
+        f1.record(stream)
+        torch.cuda.synchronize()
+        e_ms = f0.elapsed_time(f1)
+        if world > 1:
+            t = torch.tensor([e_ms], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = float(t.item())
+        e2e = {"value": total_configs * args.steps / (e_ms * 1e-3), "unit": "configs/s",
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": e_ms / args.steps}
+        del host
+
+    if rank != 0:
+        if world > 1:
+            dist.barrier()
+            dist.destroy_process_group()
+        return 0
+
+    # -------------------------------------------------------- roofline & shares
+    hbm, _, peak_src = measured_peaks()
+    phase = {"convert": 0.0, "kernel": 0.0, "backconv": 0.0, "quality": 0.0}
+    kb = kt = cb = ct = 0.0
+    speedup = {}
+    n_kernel_groups = 0
+    for a in apps:
+        arr = last[a["kind"]]
+        m = a["app"].num_objects
+        phase["convert"] += float(arr["convert_ms"].sum())
+        phase["kernel"] += float(arr["kernel_ms"].sum())
+        phase["backconv"] += float(arr["backconv_ms"].sum())
+        phase["quality"] += float(arr["quality_ms"].sum())
+        for r in arr:
+            prec = decode(int(r["config_id"]), m)
+            b = kernel_bytes(a["kind"], a["dims"], prec)
+            if b is not None:
+                kb += b
+                kt += float(r["kernel_ms"])
+                n_kernel_groups += 1
+            c = convert_bytes(a["app"].objects, prec)
+            if c:
+                cb += c
+                ct += float(r["convert_ms"])
+        f32 = arr[arr["config_id"] == (3 ** m - 1) // 2]
+        bi = D.best_index(arr)
+        if len(f32) and bi >= 0:
+            speedup[a["kind"]] = {
+                "all_f32_ms": round(float(f32["total_ms"][0]), 4),
+                "best_id": int(arr["config_id"][bi]), "best_prec": decode(int(arr["config_id"][bi]), m),
+                "best_ms": round(float(arr["total_ms"][bi]), 4),
+                "speedup": round(float(f32["total_ms"][0] / arr["total_ms"][bi]), 3),
+                "passing": int(arr["pass"].sum()), "configs": int(len(arr))}
+    roof = None
+    if kt > 0:
+        ach = kb / (kt * 1e-3) / 1e9
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        if os.path.exists(tp):
+            try:
+                traffic = json.load(open(tp)).get("kernel_group_dram_bytes")
+            except Exception:
+                traffic = None
+        roof = {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "unit": "GB/s",
+                "frac": round(ach / hbm, 4), "traffic": traffic,
+                "peak_source": peak_src + " (MEASURED_PEAKS.json hbm_gbs)" if peak_src == "measured"
+                else "fallback (B200_PROFILING.md)",
+                "kernel": "a3 mat-vec statement kernels of one configuration (rowdot/colsum/axpby)",
+                "algorithmic_bytes_per_launch": round(kb / max(n_kernel_groups, 1)),
+                "avg_launch_ms": round(kt / max(n_kernel_groups, 1), 5)}
+    conv_roof = {"achieved": round(cb / (ct * 1e-3) / 1e9, 1), "frac": round(cb / (ct * 1e-3) / 1e9 / hbm, 4)} \
+        if ct > 0 else None
+
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        cpu = cpu_baseline(args)
+
+    conv = None
+    if not args.no_conversion:
+        flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+        conv = conversion_sweep(torch, B, flush)
+        conv = {k: {"gbs": v, "frac_of_measured": round(v / hbm, 4), "frac_of_8tbs": round(v / 8000, 4)}
+                for k, v in conv.items()}
+
+    tot_phase = sum(phase.values())
+    line = {
+        "metric": "configs evaluated/s", "value": round(value, 2), "unit": "configs/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(el_ms / args.steps, 4), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None,
+        "dtype": "f64/f32/f16 (per memory object, per configuration)", "data": "synthetic",
+        "config": {"workload": args.workload,
+                   "apps": ["%s %s" % (a["kind"], "x".join(map(str, a["dims"]))) for a in apps],
+                   "configs_per_step": total_configs, "input_set": args.input_set, "toq": args.toq,
+                   "step": "a0 reference + full 3^M config space per app (a1-a7)",
+                   "l2": "inputs larger than L2 (each matrix 1 GiB fp32 > 126 MB)",
+                   "parallelism": "configs partitioned over %d GPU(s), NCCL result gather" % world},
+        "e2e": e2e, "gpu_launches": launches,
+        "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
+        "phase_share": {k: round(v / tot_phase, 4) for k, v in phase.items()} if tot_phase else None,
+        "conversion_roofline_in_sweep": conv_roof,
+        "conversion_gbs": conv,
+        "speedup_vs_fp32_at_toq": speedup,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -54,6 +54,9 @@ typedef enum {
 PS_API const char *ps_status_string(int status);
 PS_API const char *ps_last_error(void);
 PS_API const char *ps_version(void);
+/* Number of CUDA kernels this library has launched in this process (all threads).
+ * Used by bench.py to report how many of the library's kernels ran. */
+PS_API uint64_t ps_kernel_launches(void);
 
 /* ------------------------------------------------------------------------- */
 /* (1) Device-side type conversion of one memory object (Fig. 3c). */

@@ -23,7 +23,8 @@ ROLE_IN, ROLE_OUT, ROLE_INOUT, ROLE_TEMP = 0, 1, 2, 3
 
 # every symbol include/prescaler.h declares
 SYMBOLS = [
-    "ps_status_string", "ps_last_error", "ps_version", "ps_convert", "ps_quality",
+    "ps_status_string", "ps_last_error", "ps_version", "ps_kernel_launches", "ps_convert",
+    "ps_quality",
     "ps_app_create", "ps_app_destroy", "ps_app_num_objects", "ps_app_object_info",
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
@@ -80,6 +81,7 @@ def lib():
                 "ps_status_string": (ctypes.c_char_p, [ctypes.c_int]),
                 "ps_last_error": (ctypes.c_char_p, []),
                 "ps_version": (ctypes.c_char_p, []),
+                "ps_kernel_launches": (ctypes.c_uint64, []),
                 "ps_convert": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_int, ctypes.c_size_t, vp]),
                 "ps_quality": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_size_t, ctypes.c_int, vp,
                                               ctypes.POINTER(PsQualityResult)]),
@@ -120,6 +122,10 @@ def ps_last_error() -> str:
 
 def ps_version() -> str:
     return lib().ps_version().decode()
+
+
+def ps_kernel_launches() -> int:
+    return int(lib().ps_kernel_launches())
 
 
 def _check(status: int, what: str):
@@ -232,11 +238,13 @@ class App:
         arr = (vp * self.num_objects)(*[_ptr(t) if t is not None else None for t in host_inputs])
         _check(lib().ps_app_load_host(self._h, arr, _stream(stream)), "ps_app_load_host")
 
-    def reference(self, stream=None):
+    def reference(self, stream=None, refs=None):
+        """a0: the all-f64 run; fills (or allocates) one fp64 buffer per output object."""
         import torch
         dev = self.workspace.device
-        refs = [torch.empty(o["n"], dtype=torch.float64, device=dev) if o["is_output"] else None
-                for o in self.objects]
+        if refs is None:
+            refs = [torch.empty(o["n"], dtype=torch.float64, device=dev) if o["is_output"] else None
+                    for o in self.objects]
         arr = (vp * self.num_objects)(*[_ptr(t) for t in refs])
         _check(lib().ps_app_reference(self._h, arr, _stream(stream)), "ps_app_reference")
         self.ref = refs

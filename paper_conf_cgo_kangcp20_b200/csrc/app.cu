@@ -18,6 +18,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <atomic>
 #include <vector>
 
 #include "common.cuh"
@@ -37,6 +38,8 @@ ps_status cuda_status(cudaError_t e, const char *what) {
   set_error("CUDA error %d (%s) in %s", (int)e, cudaGetErrorString(e), what);
   return PS_ERR_CUDA;
 }
+static std::atomic<uint64_t> g_launches{0};
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 int num_sms() {
   static int cached[64] = {0};
   int d = 0;
@@ -384,6 +387,7 @@ const char *ps_status_string(int s) {
 }
 const char *ps_last_error(void) { return g_err; }
 const char *ps_version(void) { return "prescaler-b200 0.1 (sm_100a)"; }
+uint64_t ps_kernel_launches(void) { return g_launches.load(); }
 
 ps_status ps_app_create(const char *kind, const int64_t *dims, int ndims, const double *scalars,
                         ps_app **out) {

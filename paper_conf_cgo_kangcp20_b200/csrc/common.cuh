@@ -26,8 +26,10 @@ ps_status cuda_status(cudaError_t e, const char *what);
     if (_e != cudaSuccess) return ps::cuda_status(_e, #call); \
   } while (0)
 
+void count_launch();
 #define PS_CHECK_LAUNCH(what)                                 \
   do {                                                        \
+    ps::count_launch();                                       \
     cudaError_t _e = cudaGetLastError();                      \
     if (_e != cudaSuccess) return ps::cuda_status(_e, what);  \
   } while (0)

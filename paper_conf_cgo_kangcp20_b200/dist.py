@@ -1,0 +1,150 @@
+"""Multi-GPU configuration sweep: one process per GPU, configs partitioned,
+one NCCL gather of the fixed-size result records.
+
+Configurations are independent units, so the data path has no collective: every
+rank binds its own copy of the inputs, computes the fp64 reference itself and
+runs ``ps_sweep`` over its share.  The only exchange is an
+``all_gather_into_tensor`` of the 64-byte ``ps_result`` records (padded to the
+largest share), after which every rank holds the full table sorted by config id
+and picks the same best configuration (fastest passing, ties -> lowest id,
+reading #20).
+
+Partition: longest-processing-time-first over a deterministic cost model that
+every rank evaluates identically (no communication).  The model is the B200
+analogue of the paper's System Inspector database and
+``getExpectedTransferTime`` (Alg. 1 line 20): bytes / HBM bandwidth for
+conversions and bandwidth-bound statements, flops / pipe peak for contractions.
+"""
+from __future__ import annotations
+
+import heapq
+import os
+
+import numpy as np
+
+F64, F32, F16 = 0, 1, 2
+SIZE = {F64: 8, F32: 4, F16: 2}
+# nominal B200 rates for the cost model (only relative values matter)
+HBM_BPS = 6.5e12
+PEAK = {"tc": 1.2e15, F32: 60e12, F64: 30e12}
+
+# statement tables: ("mv", A, [objects]) = one streaming pass over object A;
+# ("mm", a, b, out, (M, N, K)) = contraction; ("ew", [objects]) = elementwise
+def _statements(kind, d):
+    if kind == "gemm":
+        return [("mm", 0, 1, 2, (d[0], d[1], d[2]))]
+    if kind == "2mm":
+        return [("mm", 0, 1, 2, (d[0], d[1], d[2])), ("mm", 2, 3, 4, (d[0], d[3], d[1]))]
+    if kind == "3mm":
+        return [("mm", 0, 1, 4, (d[0], d[1], d[2])), ("mm", 2, 3, 5, (d[1], d[3], d[4])),
+                ("mm", 4, 5, 6, (d[0], d[3], d[1]))]
+    if kind == "atax":
+        return [("mv", 0, [0, 1, 3]), ("mv", 0, [0, 3, 2])]
+    if kind == "bicg":
+        return [("mv", 0, [0, 1, 2]), ("mv", 0, [0, 3, 4])]
+    if kind == "gesummv":
+        return [("mv", 0, [0, 2, 4]), ("mv", 1, [1, 2, 3])]
+    if kind == "corr":
+        return [("mv", 0, [0, 1]), ("mv", 0, [0, 1, 2]), ("ew", [0, 1, 2]),
+                ("mm", 0, 0, 3, (d[1], d[1], d[0] / 2.0))]
+    if kind == "covar":
+        return [("mv", 0, [0, 1]), ("ew", [0, 1]), ("mm", 0, 0, 2, (d[1], d[1], d[0] / 2.0))]
+    raise KeyError(kind)
+
+
+def decode(cid: int, m: int) -> list:
+    out = []
+    for _ in range(m):
+        out.append(cid % 3)
+        cid //= 3
+    return out
+
+
+def config_cost(kind: str, dims, objects, cid: int) -> float:
+    """Predicted seconds for one configuration (deterministic, identical on all ranks)."""
+    m = len(objects)
+    p = decode(cid, m)
+    d = list(dims) if len(dims) > 1 else list(dims) * 5
+    n = [int(o["rows"]) * int(o["cols"]) for o in objects]
+    t = 0.0
+    for k, o in enumerate(objects):                      # a2 conversions
+        if o["role"] in (0, 2) and (p[k] != F32 or o["role"] == 2):
+            t += n[k] * (4 + SIZE[p[k]]) / HBM_BPS
+        if o["is_output"]:                                # a4 + a5
+            t += n[k] * (SIZE[p[k]] + 12) / HBM_BPS
+    for st in _statements(kind, d):
+        if st[0] == "mv":
+            t += n[st[1]] * SIZE[p[st[1]]] / HBM_BPS
+        elif st[0] == "ew":
+            t += sum(n[k] * SIZE[p[k]] for k in st[1]) * 2 / HBM_BPS
+        else:
+            _, a, b, out, (M, N, K) = st
+            T = F64 if F64 in (p[a], p[b], p[out]) else F32
+            peak = PEAK["tc"] if (p[a] == F16 and p[b] == F16 and T == F32) else PEAK[T]
+            t += 2.0 * M * N * K / peak
+    return t
+
+
+def lpt_partition(costs, world: int) -> list:
+    """Longest-processing-time-first: returns, per rank, the list of unit indices.
+    Deterministic: ties in cost -> lower index first; ties in load -> lower rank."""
+    order = sorted(range(len(costs)), key=lambda i: (-costs[i], i))
+    heap = [(0.0, r) for r in range(world)]
+    parts = [[] for _ in range(world)]
+    for i in order:
+        load, r = heapq.heappop(heap)
+        parts[r].append(i)
+        heapq.heappush(heap, (load + costs[i], r))
+    return [sorted(p) for p in parts]
+
+
+def partition_configs(kind, dims, objects, config_ids, world: int, rank: int) -> list:
+    costs = [config_cost(kind, dims, objects, c) for c in config_ids]
+    parts = lpt_partition(costs, world)
+    return [config_ids[i] for i in parts[rank]]
+
+
+# ------------------------------------------------------------------ gather
+RECORD_BYTES = 64
+
+
+def gather_results(local: np.ndarray, group=None, device=None) -> np.ndarray:
+    """all_gather_into_tensor of the local ps_result records (structured array with
+    64-byte items); returns the full table sorted by config_id on every rank."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    dev = device if device is not None else (
+        torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl"
+        else torch.device("cpu"))
+    cnt = torch.tensor([len(local)], dtype=torch.int64, device=dev)
+    cnts = torch.zeros(world, dtype=torch.int64, device=dev)
+    dist.all_gather_into_tensor(cnts, cnt, group=group)
+    cnts = cnts.cpu().numpy()
+    mx = int(cnts.max()) if world else 0
+    buf = np.zeros(mx * RECORD_BYTES, dtype=np.uint8)
+    raw = np.ascontiguousarray(local).view(np.uint8).reshape(-1)
+    buf[:raw.size] = raw
+    send = torch.from_numpy(buf).to(dev)
+    recv = torch.empty(world * mx * RECORD_BYTES, dtype=torch.uint8, device=dev)
+    if mx:
+        dist.all_gather_into_tensor(recv, send, group=group)
+    allb = recv.cpu().numpy().reshape(world, mx * RECORD_BYTES)
+    pieces = [allb[r, :cnts[r] * RECORD_BYTES].view(local.dtype) for r in range(world)]
+    full = np.concatenate(pieces) if pieces else local[:0]
+    return full[np.argsort(full["config_id"], kind="stable")]
+
+
+def best_index(table: np.ndarray) -> int:
+    """Fastest passing configuration, ties -> lowest id (table sorted by id); -1 if none."""
+    ok = np.flatnonzero(table["pass"] != 0)
+    if ok.size == 0:
+        return -1
+    t = table["total_ms"][ok]
+    cand = ok[t == t.min()]
+    return int(cand[np.argmin(table["config_id"][cand])])
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)),
+            int(os.environ.get("LOCAL_RANK", 0)))
