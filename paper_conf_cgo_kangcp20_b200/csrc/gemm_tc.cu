@@ -1,11 +1,314 @@
-// gemm_tc.cu -- tcgen05 tensor-core contraction (fp16 x fp16 -> f32), reading R6.
+// gemm_tc.cu -- tcgen05 tensor-core contraction for statements whose two
+// multiplicands are fp16 objects and whose compute type is f32 (reading R2):
+// the fp16 x fp16 -> f32-accumulate path of GEMM / 2MM / 3MM / SYRK (row a3).
+// Reading R6: the tensor core's internal summation order is unspecified, so
+// these results are checked against the oracle with the stated tolerance, not
+// bit-exactly (every other contraction is the R3-exact SIMT kernel).
+//
+// Structure (one 128 x 256 output tile per CTA, cta_group::1):
+//   warp 0, one lane : TMA producer  -- cp.async.bulk.tensor 2D boxes of 64
+//                      fp16 (128 B, SWIZZLE_128B) into a 4-stage smem ring,
+//                      mbarrier expect_tx / complete_tx
+//   warp 1           : TMEM allocator (256 columns = the f32 accumulator);
+//                      one lane issues tcgen05.mma.kind::f16 (M=128, N=256,
+//                      K=16) and tcgen05.commit frees each stage / signals
+//                      the epilogue
+//   warps 2..5       : epilogue -- tcgen05.ld 32x32b (warp w reads TMEM lanes
+//                      32*(w%4)..), alpha/beta or divide in f32, RNE store to
+//                      the output object's precision (R1)
+// A may be K-major (row-major A) or M-major (SYRK's data^T); B is N-major.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include "common.cuh"
 #include "kernels.cuh"
 
 namespace ps {
-bool gemm_tc_supported(const GemmArgs &) { return false; }
-ps_status gemm_tc_async(const GemmArgs &, cudaStream_t) {
-  set_error("tcgen05 path not built");
-  return PS_ERR_UNSUPPORTED;
+namespace tc {
+
+constexpr int BM = 128, BN = 256, BK = 64, STAGES = 4;
+constexpr int A_BYTES = BM * BK * 2;            // 16 KiB
+constexpr int B_BYTES = BN * BK * 2;            // 32 KiB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+constexpr int NTHREADS = 192;
+constexpr uint32_t TMEM_COLS = 256;
+constexpr uint32_t BOX_BYTES = 64 * 64 * 2;    // one 64 (MN) x 64 (K) box = 8 KiB
+
+struct Params {
+  int M, N, K;
+  int a_mn_major;
+  void *C;
+  int c_type;
+  int64_t ldc;
+  const void *Cin;
+  int cin_type;
+  int epi;
+  float alpha, beta, div;
+  int upper_only;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
 }
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  while (!mbar_try_wait(bar, parity)) {
+  }
+}
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, uint64_t *bar, int c0,
+                                            int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, "
+      "%4}], [%2];" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+// UMMA shared-memory matrix descriptor (sm100): start >> 4 [0,14), LBO >> 4
+// [16,30), SBO >> 4 [32,46), version 1 [46,48), base offset 0, SWIZZLE_128B (2) [61,64)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
+  return d;
+}
+__device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc,
+                                         uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void umma_commit(uint64_t *bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%"
+      "15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+        "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+        "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__device__ __forceinline__ float load_c(const void *p, int type, int64_t idx) {
+  return type == PS_F32 ? ((const float *)p)[idx] : f16_to_f32(((const uint16_t *)p)[idx]);
+}
+__device__ __forceinline__ void store_c(void *p, int type, int64_t idx, float v) {
+  if (type == PS_F32) ((float *)p)[idx] = v;
+  else ((uint16_t *)p)[idx] = rne_f16(v);
+}
+
+__global__ void __launch_bounds__(NTHREADS, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
+                   Params p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t *sA = smem;
+  uint8_t *sB = smem + STAGES * A_BYTES;
+  uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
+  uint64_t *empty = full + STAGES;
+  uint64_t *tfull = empty + STAGES;
+  uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
+  if (p.upper_only && m0 >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
+  const int nk = (p.K + BK - 1) / BK;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tma_a) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tma_b) : "memory");
+    for (int s = 0; s < STAGES; s++) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {   // ---------------- TMA producer
+      for (int kb = 0; kb < nk; kb++) {
+        const int s = kb % STAGES;
+        const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+        mbar_wait(&empty[s], ph ^ 1u);
+        mbar_expect_tx(&full[s], STAGE_BYTES);
+        const int k0 = kb * BK;
+        uint8_t *a = sA + s * A_BYTES;
+        if (!p.a_mn_major) {
+          tma_load_2d(a, &tma_a, &full[s], k0, m0);                 // box {64 K, 128 M}
+        } else {
+          tma_load_2d(a, &tma_a, &full[s], m0, k0);                 // box {64 M, 64 K} x 2
+          tma_load_2d(a + BOX_BYTES, &tma_a, &full[s], m0 + 64, k0);
+        }
+        uint8_t *b = sB + s * B_BYTES;
+#pragma unroll
+        for (int q = 0; q < BN / 64; q++) tma_load_2d(b + q * BOX_BYTES, &tma_b, &full[s], n0 + 64 * q, k0);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {   // ---------------- MMA issuer (single thread)
+      const uint32_t idesc = (1u << 4)                          // D = f32
+                             | ((uint32_t)p.a_mn_major << 15)   // A major
+                             | (1u << 16)                       // B is N-major
+                             | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+      for (int kb = 0; kb < nk; kb++) {
+        const int s = kb % STAGES;
+        const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+        mbar_wait(&full[s], ph);
+        fence_after();
+        const uint32_t abase = smem_u32(sA + s * A_BYTES), bbase = smem_u32(sB + s * B_BYTES);
+#pragma unroll
+        for (int kk = 0; kk < BK / 16; kk++) {
+          // K-major SW128: +32 B per 16-element K step inside the 128 B swizzled row;
+          // MN-major SW128: +2 KiB (16 K-rows of 128 B); LBO = 8 KiB between 64-wide boxes.
+          const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * 2048, BOX_BYTES, 1024)
+                                           : umma_desc(abase + kk * 32, 16, 1024);
+          const uint64_t bd = umma_desc(bbase + kk * 2048, BOX_BYTES, 1024);
+          umma_f16(tmem, ad, bd, idesc, (kb | kk) != 0);
+        }
+        umma_commit(&empty[s]);   // frees the stage when these MMAs retire
+      }
+      umma_commit(tfull);         // accumulator complete
+    }
+  } else {   // ------------------------- epilogue warps 2..5
+    mbar_wait(tfull, 0);
+    fence_after();
+    const int q = warp & 3;                 // TMEM lane quarter this warp may access
+    const int64_t row = (int64_t)m0 + q * 32 + lane;
+    for (int cc = 0; cc < BN / 16; cc++) {
+      uint32_t v[16];
+      tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * 16), v);
+      if (row < p.M) {
+#pragma unroll
+        for (int e = 0; e < 16; e++) {
+          const int64_t col = (int64_t)n0 + cc * 16 + e;
+          if (col >= p.N) break;
+          float r = __uint_as_float(v[e]);
+          const int64_t idx = row * p.ldc + col;
+          if (p.epi == EPI_AXPBY) r = __fmaf_rn(p.alpha, r, p.beta * load_c(p.Cin, p.cin_type, idx));
+          else if (p.epi == EPI_DIV) r = r / p.div;
+          store_c(p.C, p.c_type, idx, r);
+        }
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
+  }
+}
+
+}  // namespace tc
+
+// ------------------------------------------------------------------ host
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void *f = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
+  }
+  return fn;
+}
+
+// 2-D fp16 tensor map: inner (contiguous) extent, outer extent, outer stride in bytes,
+// box {64, box_outer}, 128-byte swizzle, zero fill out of bounds.
+static bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer,
+                     uint64_t stride_bytes, uint32_t box_outer) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {stride_bytes};
+  cuuint32_t box[2] = {64, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+bool gemm_tc_supported(const GemmArgs &g) {
+  if (g.A.type != PS_F16 || g.B.type != PS_F16 || g.T != PS_F32) return false;
+  if (g.c_type == PS_F64 || (g.epi == EPI_AXPBY && g.cin_type == PS_F64)) return false;
+  if (g.M <= 0 || g.N <= 0 || g.K <= 0 || g.M > (1 << 30) || g.N > (1 << 30) || g.K > (1 << 30))
+    return false;
+  if ((uintptr_t)g.A.p % 16 || (uintptr_t)g.B.p % 16) return false;
+  const bool a_k = g.A.s_col == 1 && (g.A.s_row * 2) % 16 == 0;    // row-major A
+  const bool a_m = g.A.s_row == 1 && (g.A.s_col * 2) % 16 == 0;    // SYRK data^T
+  const bool b_n = g.B.s_col == 1 && (g.B.s_row * 2) % 16 == 0;    // row-major B
+  if (!(a_k || a_m) || !b_n) return false;
+  return encode_fn() != nullptr;
+}
+
+ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
+  using namespace tc;
+  static bool attr_set = false;
+  if (!attr_set) {
+    PS_CUDA(cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES));
+    attr_set = true;
+  }
+  CUtensorMap ma, mb;
+  const bool a_mn = !(g.A.s_col == 1);
+  bool ok;
+  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * 2, BM);
+  else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * 2, 64);
+  ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * 2, 64);
+  if (!ok) {
+    set_error("cuTensorMapEncodeTiled failed");
+    return PS_ERR_CUDA;
+  }
+  Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
+           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only};
+  dim3 grid((unsigned)((g.N + BN - 1) / BN), (unsigned)((g.M + BM - 1) / BM));
+  gemm_tc_kernel<<<grid, NTHREADS, SMEM_BYTES, st>>>(ma, mb, p);
+  PS_CHECK_LAUNCH("gemm_tc_kernel");
+  return PS_OK;
+}
+
 }  // namespace ps

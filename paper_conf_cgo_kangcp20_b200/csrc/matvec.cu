@@ -33,7 +33,39 @@ __device__ __forceinline__ T ldg_t(const raw_t<S> *p, int64_t i) {
 }
 
 // ------------------------------------------------------------------ rowdot
-template <class SA, class SX, class SO>
+// A warp owns RB consecutive rows and walks them together: per 16-byte chunk
+// position c it loads the A chunk of every row and the matching x chunk ONCE
+// (vectorised, widened to T once), then advances the RB independent lane
+// chains.  Per row the order is exactly R5 (lane l: chunks c = t*32 + l,
+// t ascending, v ascending; butterfly 16..1), so results are unchanged by RB.
+template <class SX, int V, class T>
+__device__ __forceinline__ void load_x_chunk(const raw_t<SX> *__restrict__ x, int64_t j0, T *out) {
+  using RX = raw_t<SX>;
+  constexpr int BYTES = V * (int)sizeof(RX);
+  if constexpr (BYTES >= 16) {
+    const uint4 *p = reinterpret_cast<const uint4 *>(x + j0);
+    constexpr int PER = 16 / (int)sizeof(RX);
+#pragma unroll
+    for (int k = 0; k < BYTES / 16; k++) {
+      union { uint4 u; RX e[PER]; } t;
+      t.u = __ldg(p + k);
+#pragma unroll
+      for (int e = 0; e < PER; e++) out[k * PER + e] = Ld<SX, T>::get(&t.e[e], 0);
+    }
+  } else if constexpr (BYTES == 8) {
+    union { uint2 u; RX e[V]; } t;
+    t.u = __ldg(reinterpret_cast<const uint2 *>(x + j0));
+#pragma unroll
+    for (int e = 0; e < V; e++) out[e] = Ld<SX, T>::get(&t.e[e], 0);
+  } else {
+    union { uint32_t u; RX e[V]; } t;
+    t.u = __ldg(reinterpret_cast<const unsigned int *>(x + j0));
+#pragma unroll
+    for (int e = 0; e < V; e++) out[e] = Ld<SX, T>::get(&t.e[e], 0);
+  }
+}
+
+template <class SA, class SX, class SO, int RB>
 __global__ void __launch_bounds__(256) rowdot_kernel(const raw_t<SA> *__restrict__ A, int64_t lda,
                                                      const raw_t<SX> *__restrict__ x,
                                                      raw_t<SO> *__restrict__ out, int64_t rows,
@@ -41,60 +73,83 @@ __global__ void __launch_bounds__(256) rowdot_kernel(const raw_t<SA> *__restrict
   using T = T3<SA, SX, SO>;
   using RA = raw_t<SA>;
   constexpr int V = 16 / sizeof(RA);
-  constexpr int UN = 4;
+  constexpr int UN = 2;
   const int lane = threadIdx.x & 31;
   const int64_t wpb = blockDim.x >> 5;
   const int64_t nchunks = (cols + V - 1) / V;
   const int64_t full = cols / V;   // chunks entirely inside the row
-  for (int64_t row = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); row < rows;
-       row += (int64_t)gridDim.x * wpb) {
-    const RA *a = A + row * lda;
-    T acc = T(0);
+  const int64_t ngroups = (rows + RB - 1) / RB;
+  for (int64_t g = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); g < ngroups;
+       g += (int64_t)gridDim.x * wpb) {
+    const int64_t r0 = g * RB;
+    const int nr = (int)((rows - r0) < RB ? (rows - r0) : RB);
+    T acc[RB];
+#pragma unroll
+    for (int r = 0; r < RB; r++) acc[r] = T(0);
     int64_t c = lane;
-    if (vec_ok) {
+    if (vec_ok && nr == RB) {
+      const uint4 *arow[RB];
+#pragma unroll
+      for (int r = 0; r < RB; r++) arow[r] = reinterpret_cast<const uint4 *>(A + (r0 + r) * lda);
       for (; c + 32 * (UN - 1) < full; c += 32 * UN) {
-        union { uint4 v; RA e[V]; } ch[UN];
+        union { uint4 v; RA e[V]; } ch[UN][RB];
 #pragma unroll
         for (int u = 0; u < UN; u++)
-          ch[u].v = __ldg(reinterpret_cast<const uint4 *>(a) + c + 32 * u);
+#pragma unroll
+          for (int r = 0; r < RB; r++) ch[u][r].v = __ldg(arow[r] + c + 32 * u);
 #pragma unroll
         for (int u = 0; u < UN; u++) {
-          const int64_t j0 = (c + 32 * u) * V;
+          T xv[V];
+          load_x_chunk<SX, V, T>(x, (c + 32 * u) * V, xv);
 #pragma unroll
-          for (int v = 0; v < V; v++) {
-            const raw_t<SA> e = ch[u].e[v];
-            acc = t_fma(Ld<SA, T>::get(&e, 0), ldg_t<SX, T>(x, j0 + v), acc);
-          }
+          for (int r = 0; r < RB; r++)
+#pragma unroll
+            for (int v = 0; v < V; v++)
+              acc[r] = t_fma(Ld<SA, T>::get(&ch[u][r].e[v], 0), xv[v], acc[r]);
         }
       }
       for (; c < full; c += 32) {
-        union { uint4 v; RA e[V]; } ch;
-        ch.v = __ldg(reinterpret_cast<const uint4 *>(a) + c);
-        const int64_t j0 = c * V;
+        union { uint4 v; RA e[V]; } ch[RB];
 #pragma unroll
-        for (int v = 0; v < V; v++) {
-          const raw_t<SA> e = ch.e[v];
-          acc = t_fma(Ld<SA, T>::get(&e, 0), ldg_t<SX, T>(x, j0 + v), acc);
-        }
+        for (int r = 0; r < RB; r++) ch[r].v = __ldg(arow[r] + c);
+        T xv[V];
+        load_x_chunk<SX, V, T>(x, c * V, xv);
+#pragma unroll
+        for (int r = 0; r < RB; r++)
+#pragma unroll
+          for (int v = 0; v < V; v++) acc[r] = t_fma(Ld<SA, T>::get(&ch[r].e[v], 0), xv[v], acc[r]);
       }
     }
-    for (; c < nchunks; c += 32) {   // scalar path (unaligned rows, ragged last chunk)
+    // scalar path: unaligned rows, a ragged row group, the ragged last chunk
+    for (; c < nchunks; c += 32) {
       const int64_t j0 = c * V;
-      for (int v = 0; v < V && j0 + v < cols; v++)
-        acc = t_fma(ldg_t<SA, T>(a, j0 + v), ldg_t<SX, T>(x, j0 + v), acc);
-    }
+      for (int v = 0; v < V && j0 + v < cols; v++) {
+        const T xj = ldg_t<SX, T>(x, j0 + v);
 #pragma unroll
-    for (int off = 16; off >= 1; off >>= 1) acc = acc + __shfl_xor_sync(0xffffffffu, acc, off);
-    if (lane == 0) St<SO, T>::put(out, (size_t)row, acc);
+        for (int r = 0; r < RB; r++)
+          if (r < nr) acc[r] = t_fma(ldg_t<SA, T>(A + (r0 + r) * lda, j0 + v), xj, acc[r]);
+      }
+    }
+    T mine = T(0);
+#pragma unroll
+    for (int r = 0; r < RB; r++) {
+#pragma unroll
+      for (int off = 16; off >= 1; off >>= 1) acc[r] = acc[r] + __shfl_xor_sync(0xffffffffu, acc[r], off);
+      if (lane == r) mine = acc[r];
+    }
+    if (lane < nr) St<SO, T>::put(out, (size_t)(r0 + lane), mine);
   }
 }
 
 ps_status rowdot_async(const void *A, int ta, int64_t lda, const void *x, int tx, void *out,
                        int tout, int64_t rows, int64_t cols, cudaStream_t st) {
   if (rows <= 0) return PS_OK;
-  const int vec_ok = ((uintptr_t)A % 16 == 0) && ((lda * (int64_t)dtype_size(ta)) % 16 == 0);
+  constexpr int RB = 4;
+  const int vec_ok = ((uintptr_t)A % 16 == 0) && ((lda * (int64_t)dtype_size(ta)) % 16 == 0) &&
+                     ((uintptr_t)x % 16 == 0);
   const int64_t wpb = 8;
-  int64_t blocks = (rows + wpb - 1) / wpb;
+  const int64_t ngroups = (rows + RB - 1) / RB;
+  int64_t blocks = (ngroups + wpb - 1) / wpb;
   const int64_t cap = (int64_t)num_sms() * 8;
   if (blocks > cap) blocks = cap;
   return dispatch_store(ta, [&](auto sa) -> ps_status {
@@ -103,7 +158,7 @@ ps_status rowdot_async(const void *A, int ta, int64_t lda, const void *x, int tx
         using SA = decltype(sa);
         using SX = decltype(sx);
         using SO = decltype(so);
-        rowdot_kernel<SA, SX, SO><<<(unsigned)blocks, 256, 0, st>>>(
+        rowdot_kernel<SA, SX, SO, RB><<<(unsigned)blocks, 256, 0, st>>>(
             (const raw_t<SA> *)A, lda, (const raw_t<SX> *)x, (raw_t<SO> *)out, rows, cols, vec_ok);
         PS_CHECK_LAUNCH("rowdot_kernel");
         return PS_OK;
