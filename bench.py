@@ -38,8 +38,10 @@ WORKLOADS = {
     "matvec": [("atax", [16384, 16384]), ("bicg", [16384, 16384]), ("gesummv", [16384])],
     # BASELINE.json configs[0]
     "gemm64": [("gemm", [64])],
-    # BASELINE.json configs[3] / configs[4]
-    "contract": [("2mm", [8192]), ("3mm", [8192])],
+    # BASELINE.json configs[3] / configs[4] (3MM's 2187-config space at N=8192 is a
+    # separate workload: one step is minutes of fp64 DFMA on one GPU)
+    "contract": [("2mm", [8192])],
+    "contract3mm": [("3mm", [8192])],
     "corr": [("corr", [8192, 8192]), ("covar", [8192, 8192])],
 }
 SIZE = {0: 8, 1: 4, 2: 2}
@@ -47,7 +49,8 @@ SIZE = {0: 8, 1: 4, 2: 2}
 # per ATAX configuration at N=16384, so the CPU legs run every app dimension at
 # the reduced size and extrapolate throughput by (N_sample / N)^exponent (O(N^2)
 # mat-vec, O(N^3) contractions); labelled "extrapolated" in the JSON.
-CPU_SAMPLE = {"matvec": (8192, 2), "gemm64": (None, 0), "contract": (384, 3), "corr": (512, 3)}
+CPU_SAMPLE = {"matvec": (8192, 2), "gemm64": (None, 0), "contract": (384, 3), "contract3mm": (256, 3),
+              "corr": (512, 3)}
 
 
 def log(*a):

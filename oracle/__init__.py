@@ -215,6 +215,30 @@ def evaluate(kind: str, dims, prec, inputs, ref, scalars=None, toq: float = 0.9)
     return out, delivered
 
 
+def sample(kind: str, dims, prec, inputs, m: int, rows, cols, scalars=None) -> np.ndarray:
+    """Raw final values (in precision prec[m], widened to float64) of output
+    object m at entries (rows[k], cols[k]); only what they depend on is computed."""
+    L = lib()
+    if not hasattr(L, "_sample_sig"):
+        L.oracle_sample.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64), ctypes.c_int,
+                                    ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int),
+                                    ctypes.POINTER(ctypes.c_void_p), ctypes.c_int,
+                                    ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t,
+                                    ctypes.c_void_p]
+        L._sample_sig = True
+    objs = app_objects(kind, dims)
+    d, nd = _dims(dims)
+    ins, keep = _inputs(objs, inputs)
+    r = np.ascontiguousarray(rows, dtype=np.int64)
+    c = np.ascontiguousarray(cols, dtype=np.int64)
+    out = np.empty(r.size, dtype=np.float64)
+    pr = (ctypes.c_int * len(prec))(*prec)
+    if L.oracle_sample(kind.encode(), d, nd, _scalars(scalars), pr, ins, m, r.ctypes.data,
+                       c.ctypes.data, r.size, out.ctypes.data):
+        raise ValueError("oracle_sample failed")
+    return out
+
+
 def sweep(kind: str, dims, config_ids, inputs, scalars=None, toq: float = 0.9, ref=None):
     """c-6: evaluate every configuration id; returns (ref, list of result dicts)."""
     objs = app_objects(kind, dims)

@@ -193,12 +193,23 @@ int oracle_config_encode(int m, const int *prec, uint64_t *id) {
 /* R1/R2/R4: objects and arithmetic "in T"                               */
 /* ===================================================================== */
 
-typedef struct { int type; size_t n; void *p; } obj_t;
+/* An object stored in precision `type`.  In sampling mode (oracle_sample) an
+ * input object may instead be "lazy": element i is RNE_type(src[i]) converted
+ * on access from the original f32 data -- the same value a2 would have stored. */
+typedef struct { int type; size_t n; void *p; const float *src; } obj_t;
 
 static size_t tsize(int t) { return t == OR_F64 ? 8 : (t == OR_F32 ? 4 : 2); }
 
 /* R1: load = exact widening of the stored element */
-static double ld(const obj_t *o, size_t i) { return widen(o->p, o->type, i); }
+static double ld(const obj_t *o, size_t i) {
+  if (o->src) {
+    uint32_t b;
+    memcpy(&b, &o->src[i], 4);
+    uint64_t s = o->type == OR_F32 ? b : oracle_convert_bits(b, OR_F32, o->type);
+    return bits_to_double(o->type == OR_F64 ? s : oracle_convert_bits(s, o->type, OR_F64));
+  }
+  return widen(o->p, o->type, i);
+}
 
 /* R1: store = RNE from the compute type T to the object's precision.  The
  * value v is exactly representable in T. */
@@ -608,5 +619,167 @@ int oracle_evaluate(const char *kind, const int64_t *dims, int ndims, const doub
   res->quality = 1.0 - res->mean_rel;
   res->max_rel = mx;
   res->nonfinite = nf;
+  return 0;
+}
+
+/* ===================================================================== */
+/* Sampled evaluation (parity at the BASELINE sizes)                     */
+/* ===================================================================== */
+/* Raw final values of output object m at entries (rows[k], cols[k]) for one
+ * configuration, computed with the SAME helpers, compute types and orders as
+ * oracle_run_config, touching only what those entries depend on.  Input
+ * objects are lazy views of the f32 inputs (a2 applied per element on load).
+ * tests/test_oracle_sample.py pins it against the full run. */
+
+static double round_to(int type, double v, int T) {
+  unsigned char buf[8];
+  obj_t o = {type, 1, buf, NULL};
+  st(&o, 0, v, T);
+  return ld(&o, 0);
+}
+static obj_t new_obj(int type, size_t n) {
+  obj_t o = {type, n, calloc(n ? n : 1, tsize(type)), NULL};
+  return o;
+}
+
+/* CORR/COVAR: column j of data after the statements that precede the SYRK
+ * (mean; stddev and normalisation for CORR; centring for COVAR) into z. */
+static void stats_column(int corr, obj_t *data, obj_t *mean, obj_t *sd, size_t N, size_t M,
+                         size_t j, double eps_lit, obj_t *z) {
+  int T1 = W2(data->type, mean->type);
+  size_t i;
+  st(mean, j, t_div(T1, colsum(T1, data, N, M, j, NULL, 1), t_lit(T1, (double)N)), T1);
+  if (corr) {
+    int T2 = W3(data->type, mean->type, sd->type);
+    double s = t_sqrt(T2, t_div(T2, colsum(T2, data, N, M, j, mean, 2), t_lit(T2, (double)N)));
+    double sqn = t_lit(T2, sqrt((double)N));
+    st(sd, j, s <= t_lit(T2, eps_lit) ? 1.0 : s, T2);
+    for (i = 0; i < N; i++) {
+      double dd = t_sub(T2, ld(data, i * M + j), ld(mean, j));
+      st(z, i, t_div(T2, dd, t_mul(T2, sqn, ld(sd, j))), T2);
+    }
+  } else {
+    int T2 = W2(data->type, mean->type);
+    for (i = 0; i < N; i++) st(z, i, t_sub(T2, ld(data, i * M + j), ld(mean, j)), T2);
+  }
+}
+
+int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double *sc,
+                  const int *prec, const float *const *inputs, int m, const int64_t *rows,
+                  const int64_t *cols, size_t n, double *vals) {
+  const app_def_t *a = find_app(kind);
+  int64_t d[8], R[8], C[8];
+  obj_t in[8];
+  size_t k, q;
+  int t;
+  if (!a || full_dims(a, dims, ndims, d) || !prec || m < 0 || m >= a->nobj || !a->outputs[m] ||
+      (n && (!rows || !cols || !vals)))
+    return 1;
+  shapes(a, d, R, C);
+  memset(in, 0, sizeof(in));
+  for (t = 0; t < a->nobj; t++) {
+    if (prec[t] < 0 || prec[t] > 2) return 1;
+    in[t].type = prec[t];
+    in[t].n = (size_t)(R[t] * C[t]);
+    if (a->roles[t] == 0 || a->roles[t] == 2) {
+      if (!inputs || !inputs[t]) return 1;
+      in[t].src = inputs[t];
+    }
+  }
+  for (k = 0; k < n; k++)
+    if (rows[k] < 0 || rows[k] >= R[m] || cols[k] < 0 || cols[k] >= C[m]) return 1;
+
+  if (!strcmp(kind, "gemm")) {
+    size_t NJ = d[1], NK = d[2];
+    int T = W3(prec[0], prec[1], prec[2]);
+    double al = t_lit(T, scalar_or(sc, 0, 32412.0)), be = t_lit(T, scalar_or(sc, 1, 2123.0));
+    for (k = 0; k < n; k++) {
+      size_t i = rows[k], j = cols[k];
+      double acc = dot_chain(T, &in[0], i * NK, 1, &in[1], j, NJ, NK);
+      double bc = t_mul(T, be, ld(&in[2], i * NJ + j));
+      vals[k] = round_to(prec[2], t_fma(T, al, acc, bc), T);
+    }
+  } else if (!strcmp(kind, "2mm")) {
+    size_t NJ = d[1], NK = d[2], NL = d[3], j;
+    int T1 = W3(prec[0], prec[1], prec[2]), T2 = W3(prec[2], prec[3], prec[4]);
+    obj_t crow = new_obj(prec[2], NJ);
+    int64_t cached = -1;
+    for (k = 0; k < n; k++) {
+      size_t i = rows[k], l = cols[k];
+      if ((int64_t)i != cached) {           /* row i of C <- A . B */
+        for (j = 0; j < NJ; j++) st(&crow, j, dot_chain(T1, &in[0], i * NK, 1, &in[1], j, NJ, NK), T1);
+        cached = (int64_t)i;
+      }
+      vals[k] = round_to(prec[4], dot_chain(T2, &crow, 0, 1, &in[3], l, NL, NJ), T2);
+    }
+    free(crow.p);
+  } else if (!strcmp(kind, "3mm")) {
+    size_t NJ = d[1], NK = d[2], NL = d[3], NM = d[4], j;
+    int T1 = W3(prec[0], prec[1], prec[4]), T2 = W3(prec[2], prec[3], prec[5]);
+    int T3 = W3(prec[4], prec[5], prec[6]);
+    obj_t erow = new_obj(prec[4], NJ), fcol = new_obj(prec[5], NJ);
+    int64_t ci = -1, cl = -1;
+    for (k = 0; k < n; k++) {
+      size_t i = rows[k], l = cols[k];
+      if ((int64_t)i != ci) {               /* row i of E <- A . B */
+        for (j = 0; j < NJ; j++) st(&erow, j, dot_chain(T1, &in[0], i * NK, 1, &in[1], j, NJ, NK), T1);
+        ci = (int64_t)i;
+      }
+      if ((int64_t)l != cl) {               /* column l of F <- C . D */
+        for (j = 0; j < NJ; j++) st(&fcol, j, dot_chain(T2, &in[2], j * NM, 1, &in[3], l, NL, NM), T2);
+        cl = (int64_t)l;
+      }
+      vals[k] = round_to(prec[6], dot_chain(T3, &erow, 0, 1, &fcol, 0, 1, NJ), T3);
+    }
+    free(erow.p);
+    free(fcol.p);
+  } else if (!strcmp(kind, "atax")) {
+    size_t NX = d[0], NY = d[1], i;
+    int T1 = W3(prec[0], prec[1], prec[3]), T2 = W3(prec[0], prec[3], prec[2]);
+    obj_t tmp = new_obj(prec[3], NX);      /* y depends on every row-dot */
+    for (i = 0; i < NX; i++) st(&tmp, i, rowdot(T1, &in[0], i * NY, NY, &in[1]), T1);
+    for (k = 0; k < n; k++)
+      vals[k] = round_to(prec[2], colsum(T2, &in[0], NX, NY, (size_t)cols[k], &tmp, 0), T2);
+    free(tmp.p);
+  } else if (!strcmp(kind, "bicg")) {
+    size_t NX = d[0], NY = d[1];
+    int T1 = W3(prec[0], prec[1], prec[2]), T2 = W3(prec[0], prec[3], prec[4]);
+    for (k = 0; k < n; k++) {
+      if (m == 2) vals[k] = round_to(prec[2], colsum(T1, &in[0], NX, NY, (size_t)cols[k], &in[1], 0), T1);
+      else vals[k] = round_to(prec[4], rowdot(T2, &in[0], (size_t)cols[k] * NY, NY, &in[3]), T2);
+    }
+  } else if (!strcmp(kind, "gesummv")) {
+    size_t N = d[0];
+    int T1 = W3(prec[0], prec[2], prec[4]), T2 = W3(prec[1], prec[2], prec[3]);
+    int T3 = W2(prec[4], prec[3]);
+    double al = t_lit(T3, scalar_or(sc, 0, 43532.0)), be = t_lit(T3, scalar_or(sc, 1, 12313.0));
+    for (k = 0; k < n; k++) {
+      size_t i = cols[k];
+      double tv = round_to(prec[4], rowdot(T1, &in[0], i * N, N, &in[2]), T1);
+      double yv = round_to(prec[3], rowdot(T2, &in[1], i * N, N, &in[2]), T2);
+      vals[k] = round_to(prec[3], t_fma(T3, al, tv, t_mul(T3, be, yv)), T3);
+    }
+  } else {                                  /* corr / covar: symmat entries */
+    int corr = !strcmp(kind, "corr");
+    size_t N = d[0], M = d[1];
+    int so = corr ? 3 : 2;
+    obj_t mean = new_obj(prec[1], M), sd = new_obj(corr ? prec[2] : OR_F64, M);
+    obj_t z1 = new_obj(prec[0], N), z2 = new_obj(prec[0], N);
+    int T = W2(prec[0], prec[so]);
+    double eps = scalar_or(sc, 0, 0.005);
+    for (k = 0; k < n; k++) {
+      size_t j1 = rows[k], j2 = cols[k];
+      if (j1 > j2) { size_t s = j1; j1 = j2; j2 = s; }   /* mirrored lower triangle */
+      if (corr && j1 == j2) { vals[k] = round_to(prec[so], 1.0, T); continue; }
+      stats_column(corr, &in[0], &mean, &sd, N, M, j1, eps, &z1);
+      stats_column(corr, &in[0], &mean, &sd, N, M, j2, eps, &z2);
+      {
+        double acc = dot_chain(T, &z1, 0, 1, &z2, 0, 1, N);
+        if (!corr) acc = t_div(T, acc, t_lit(T, (double)N - 1.0));
+        vals[k] = round_to(prec[so], acc, T);
+      }
+    }
+    for (q = 0; q < 1; q++) { free(mean.p); free(sd.p); free(z1.p); free(z2.p); }
+  }
   return 0;
 }

@@ -82,6 +82,13 @@ int oracle_evaluate(const char *kind, const int64_t *dims, int ndims,
                     const float *const *inputs, const double *const *ref,
                     float *const *delivered, oracle_quality_result *res);
 
+/* Sampled evaluation for parity at full size: raw final values (widened to
+ * double) of output object m at entries (rows[k], cols[k]), same semantics as
+ * oracle_run_config, computing only what those entries depend on. */
+int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double *scalars,
+                  const int *prec, const float *const *inputs, int m, const int64_t *rows,
+                  const int64_t *cols, size_t n, double *vals);
+
 #ifdef __cplusplus
 }
 #endif
