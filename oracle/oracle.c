@@ -266,27 +266,37 @@ static double dot_chain(int T, const obj_t *A, size_t ai, size_t ask,
   return acc;
 }
 
-/* R5 row-dot: y = sum_j A[row, j] x_j for a row of length n.  Lane l of 32
- * owns the 16-byte chunks c = t*32 + l (V = 16 / sizeof(stored A) elements
- * each) and runs an fma chain over them (t ascending, then v ascending).
- * Lanes then combine by xor butterfly with offsets 16,8,4,2,1 as a + partner. */
+/* R5 row-dot: y = sum_j A[row, j] x_j for a row of length n, hierarchically:
+ *  - chunk: lane l of a 32-lane slab owns the V = 16 / sizeof(stored A)
+ *    consecutive elements j = 32*V*s + l*V + v and runs an fma chain over them
+ *    from +0 (v ascending; elements past n are skipped);
+ *  - slab s (32*V columns): the 32 lane values combine by xor butterfly with
+ *    offsets 16,8,4,2,1 as a + partner;
+ *  - tile (ORACLE_ROWDOT_TILE slabs): slab sums added left to right;
+ *  - row: tile sums added left to right. */
 static double rowdot(int T, const obj_t *A, size_t row0, size_t n, const obj_t *x) {
   double lane[ORACLE_ROWDOT_LANES], nxt[ORACLE_ROWDOT_LANES];
-  size_t V = 16 / tsize(A->type), nchunks = (n + V - 1) / V, c, v;
+  size_t V = 16 / tsize(A->type), W = ORACLE_ROWDOT_LANES * V;
+  size_t nslab = (n + W - 1) / W, s, v;
+  double total = 0.0, tile = 0.0;
   int l, off;
-  for (l = 0; l < ORACLE_ROWDOT_LANES; l++) lane[l] = 0.0;
-  for (c = 0; c < nchunks; c++) {
-    l = (int)(c % ORACLE_ROWDOT_LANES);
-    for (v = 0; v < V && c * V + v < n; v++) {
-      size_t j = c * V + v;
-      lane[l] = t_fma(T, ld(A, row0 + j), ld(x, j), lane[l]);
+  for (s = 0; s < nslab; s++) {
+    for (l = 0; l < ORACLE_ROWDOT_LANES; l++) {
+      lane[l] = 0.0;
+      for (v = 0; v < V; v++) {
+        size_t j = s * W + (size_t)l * V + v;
+        if (j < n) lane[l] = t_fma(T, ld(A, row0 + j), ld(x, j), lane[l]);
+      }
     }
+    for (off = ORACLE_ROWDOT_LANES / 2; off >= 1; off >>= 1) {
+      for (l = 0; l < ORACLE_ROWDOT_LANES; l++) nxt[l] = t_add(T, lane[l], lane[l ^ off]);
+      memcpy(lane, nxt, sizeof(lane));
+    }
+    tile = (s % ORACLE_ROWDOT_TILE == 0) ? lane[0] : t_add(T, tile, lane[0]);
+    if (s % ORACLE_ROWDOT_TILE == ORACLE_ROWDOT_TILE - 1 || s == nslab - 1)
+      total = (s < ORACLE_ROWDOT_TILE) ? tile : t_add(T, total, tile);
   }
-  for (off = ORACLE_ROWDOT_LANES / 2; off >= 1; off >>= 1) {
-    for (l = 0; l < ORACLE_ROWDOT_LANES; l++) nxt[l] = t_add(T, lane[l], lane[l ^ off]);
-    memcpy(lane, nxt, sizeof(lane));
-  }
-  return lane[0];
+  return total;
 }
 
 /* R5 column-sum: z_j = sum_i A_ij w_i.  Rows are split into chunks of

@@ -50,7 +50,8 @@ int oracle_config_encode(int num_objects, const int *prec, uint64_t *id);
 
 /* ---- c-4: applications ------------------------------------------------ */
 /* Reduction-order parameters (R5).  They are part of the definition. */
-#define ORACLE_ROWDOT_LANES 32   /* lanes per row-dot warp                   */
+#define ORACLE_ROWDOT_LANES 32   /* lanes per row-dot slab                   */
+#define ORACLE_ROWDOT_TILE 8     /* slabs per row-dot tile                   */
 #define ORACLE_COLSUM_CHUNK 256  /* rows per column-sum chunk                */
 
 typedef struct {

@@ -172,6 +172,20 @@ def test_colsum_chunk_tail_exact(oracle_lib):
     assert np.array_equal(fin[2].astype(np.float64), ref[2])
 
 
+def test_rowdot_slab_and_tile_tails_exact(oracle_lib):
+    """Rows spanning several 8-slab tiles with a ragged last slab, every precision
+    of A: exact integer results (no dropped or duplicated slab/tile)."""
+    dims = [9, 8 * 32 * 8 * 2 + 3 * 32 + 5]     # > 2 f16 tiles, > 4 f32 tiles, > 8 f64 tiles
+    objs = oracle.app_objects("atax", dims)
+    rng = np.random.default_rng(13)
+    ins = _exact_ints("atax", dims, objs, rng, 0, 4)
+    ref = numpy_ref("atax", ins, objs)
+    for pa in (F64, F32, F16):
+        fin = oracle.run_config("atax", dims, [pa, F32, F64, F64], ins)
+        assert np.array_equal(fin[3].astype(np.float64), ref[3]), pa
+        assert np.array_equal(fin[2].astype(np.float64), ref[2]), pa
+
+
 # ---------------------------------------------------------- error bounds
 @pytest.mark.parametrize("kind", ["gemm", "atax", "bicg", "gesummv", "2mm"])
 def test_all_f32_within_gamma_bound(oracle_lib, kind):
