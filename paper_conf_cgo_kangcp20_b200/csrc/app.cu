@@ -153,7 +153,8 @@ void layout(ps_app *a) {
   }
   size_t pb = 0;
   if (a->kind == K_ATAX || a->kind == K_BICG || a->kind == K_CORR || a->kind == K_COVAR)
-    pb = colsum_partial_bytes(a->d[0], a->d[1]);
+    pb = tile_partial_bytes(a->d[0], a->d[1]);
+  if (a->kind == K_GESUMMV) pb = tile_partial_bytes(a->d[0], a->d[0]);
   a->partial_off = off;
   off = align_up(off + pb, 256);
   int nout = 0;
@@ -240,18 +241,17 @@ ps_status run_statements(Ctx &c) {
       S_(matmul(c, 4, 5, 6, d[0], d[3], d[1]));   // G <- E.F
       break;
     case K_ATAX:   // tmp <- A x ; y <- A^T tmp
-      S_(rowdot_async(P[0], p[0], d[1], P[1], p[1], P[3], p[3], d[0], d[1], c.st));
+      S_(rowdot_async(P[0], p[0], d[1], P[1], p[1], P[3], p[3], d[0], d[1], partial, c.st));
       S_(colsum_async(P[0], p[0], d[1], P[3], p[3], P[2], p[2], d[0], d[1],
                       compute_type({p[0], p[3], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st));
       break;
-    case K_BICG:   // s <- A^T r ; q <- A p
-      S_(colsum_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], d[0], d[1],
-                      compute_type({p[0], p[1], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st));
-      S_(rowdot_async(P[0], p[0], d[1], P[3], p[3], P[4], p[4], d[0], d[1], c.st));
+    case K_BICG:   // s <- A^T r ; q <- A p   (one pass over A)
+      S_(bicg_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], P[3], p[3], P[4], p[4], d[0], d[1],
+                    partial, c.st));
       break;
     case K_GESUMMV:   // tmp <- A x ; y <- B x ; y <- alpha tmp + beta y
-      S_(rowdot_async(P[0], p[0], d[0], P[2], p[2], P[4], p[4], d[0], d[0], c.st));
-      S_(rowdot_async(P[1], p[1], d[0], P[2], p[2], P[3], p[3], d[0], d[0], c.st));
+      S_(rowdot_async(P[0], p[0], d[0], P[2], p[2], P[4], p[4], d[0], d[0], partial, c.st));
+      S_(rowdot_async(P[1], p[1], d[0], P[2], p[2], P[3], p[3], d[0], d[0], partial, c.st));
       S_(axpby_async(P[4], p[4], P[3], p[3], d[0], a->sc[0], a->sc[1], c.st));
       break;
     case K_CORR: {

@@ -52,17 +52,21 @@ ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st);
 ps_status mirror_async(void *S, int type, int64_t M, int diag_one, cudaStream_t st);
 
 // ------------------------------------------------------------ mat-vec (a3)
-constexpr int ROWDOT_LANES = 32;     // R5
-constexpr int COLSUM_CHUNK = 256;    // R5
-// out[i] = RNE_out( butterfly( lane fma chains ) ), R5 row-dot
+constexpr int COLSUM_CHUNK = 256;    // R5: rows per column-sum chunk
+// workspace for the chunk / tile partials of one statement on a rows x cols matrix
+size_t tile_partial_bytes(int64_t rows, int64_t cols);
+// out[i] = RNE_out(row-dot of row i), R5 hierarchical order (tiles.cu)
 ps_status rowdot_async(const void *A, int ta, int64_t lda, const void *x, int tx, void *out,
-                       int tout, int64_t rows, int64_t cols, cudaStream_t st);
+                       int tout, int64_t rows, int64_t cols, void *partial, cudaStream_t st);
+// BICG in ONE pass over A: s = A^T r (column sums), q = A p (row dots)
+ps_status bicg_async(const void *A, int ta, int64_t lda, const void *r, int tr, void *s, int ts,
+                     const void *p, int tp, void *q, int tq, int64_t rows, int64_t cols,
+                     void *partial, cudaStream_t st);
 // column sums over 256-row chunks:
 //   mode 0: p = fma(A_ij, w_i, p)   mode 1: p = p + A_ij   mode 2: d = A_ij - w_j, p = fma(d, d, p)
 // finalize: 0 plain, 1 total / n, 2 stddev (sqrt(total / n), <= eps -> 1)
 enum ColMode { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
 enum ColFin { FIN_PLAIN = 0, FIN_MEAN = 1, FIN_STDDEV = 2 };
-size_t colsum_partial_bytes(int64_t rows, int64_t cols);
 ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
                        int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
                        double eps, void *partial, cudaStream_t st);
