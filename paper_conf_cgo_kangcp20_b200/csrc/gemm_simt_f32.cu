@@ -1,0 +1,21 @@
+// gemm_simt_f32.cu -- instantiations of the R3-exact SIMT contraction with
+// compute type f32 (operands stored in f32 or f16; FFMA chains).
+#include "gemm_simt.cuh"
+
+namespace ps {
+namespace simt {
+
+ps_status gemm_simt_f32(const GemmArgs &g, cudaStream_t st) {
+  const Params p = make_params(g);
+  const bool ak = g.A.s_col == 1;
+  auto pick = [&](auto sa) -> ps_status {
+    using SA = decltype(sa);
+    if (g.B.type == PS_F16) return launch<float, SA, F16>(p, ak, g.alpha, g.beta, g.div, st);
+    return launch<float, SA, float>(p, ak, g.alpha, g.beta, g.div, st);
+  };
+  if (g.A.type == PS_F16) return pick(F16());
+  return pick(float());
+}
+
+}  // namespace simt
+}  // namespace ps
