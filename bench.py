@@ -127,6 +127,55 @@ def kernel_bytes(kind, dims, prec):
     return None
 
 
+# contraction statements: (a, b, out, M, N, K-flop-factor); SYRK computes the
+# upper triangle only, so its algorithmic work is M*M*N multiply-adds / 2 * 2.
+def _contractions(kind, d):
+    if kind == "gemm":
+        return [(0, 1, 2, d[0], d[1], d[2])]
+    if kind == "2mm":
+        return [(0, 1, 2, d[0], d[1], d[2]), (2, 3, 4, d[0], d[3], d[1])]
+    if kind == "3mm":
+        return [(0, 1, 4, d[0], d[1], d[2]), (2, 3, 5, d[1], d[3], d[4]), (4, 5, 6, d[0], d[3], d[1])]
+    if kind in ("corr", "covar"):
+        return [(0, 0, 3 if kind == "corr" else 2, d[1], d[1], d[0] / 2.0)]
+    return []
+
+
+def contraction_roofline(apps, last):
+    """a3 of contraction workloads: frac = sum of ideal statement times (flops / the
+    peak of the pipe the statement runs on) / sum of measured kernel times.  Peaks:
+    tensor = MEASURED_PEAKS bf16 burst (fp16 has the same dense rate); FFMA / DFMA
+    derived from unit counts (128 / 64 per SM per clock) x 148 SMs x 1965 MHz."""
+    _, tc_peak, _ = measured_peaks()
+    peaks = {"tensor": tc_peak, 1: 148 * 128 * 2 * 1.965e9 / 1e12, 0: 148 * 64 * 2 * 1.965e9 / 1e12}
+    ideal = meas = flops = 0.0
+    paths = {}
+    for a in apps:
+        dims = a["dims"] if len(a["dims"]) > 1 else a["dims"] * 5
+        sts = _contractions(a["kind"], dims)
+        if not sts:
+            return None
+        m = a["app"].num_objects
+        for r in last[a["kind"]]:
+            p = decode(int(r["config_id"]), m)
+            for (x, y, o, M, N, K) in sts:
+                T = 0 if 0 in (p[x], p[y], p[o]) else 1
+                path = "tensor" if (p[x] == 2 and p[y] == 2 and T == 1) else T
+                f = 2.0 * M * N * K
+                flops += f
+                ideal += f / (peaks[path] * 1e12)
+                paths[str(path)] = paths.get(str(path), 0) + 1
+            meas += float(r["kernel_ms"]) * 1e-3
+    if meas <= 0:
+        return None
+    return {"bound": "tensor+fma", "achieved": round(flops / meas / 1e12, 2), "unit": "TFLOP/s",
+            "peak": {"tensor": tc_peak, "ffma": round(peaks[1], 1), "dfma": round(peaks[0], 1)},
+            "frac": round(ideal / meas, 4), "traffic": None,
+            "peak_source": "tensor: MEASURED_PEAKS.json bf16_tflops (burst); FMA pipes derived",
+            "kernel": "a3 contraction statements (gemm_tc_kernel / gemm_simt_kernel)",
+            "statements_by_path": paths}
+
+
 def convert_bytes(objects, prec):
     b = 0
     for o, p in zip(objects, prec):
@@ -423,25 +472,42 @@ def main():
                 "best_ms": round(float(arr["total_ms"][bi]), 4),
                 "speedup": round(float(f32["total_ms"][0] / arr["total_ms"][bi]), 3),
                 "passing": int(arr["pass"].sum()), "configs": int(len(arr))}
-    roof = None
-    if kt > 0:
-        ach = kb / (kt * 1e-3) / 1e9
-        traffic = None
-        tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-        if os.path.exists(tp):
-            try:
-                traffic = json.load(open(tp)).get("kernel_group_dram_bytes")
-            except Exception:
-                traffic = None
-        roof = {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "unit": "GB/s",
-                "frac": round(ach / hbm, 4), "traffic": traffic,
-                "peak_source": peak_src + " (MEASURED_PEAKS.json hbm_gbs)" if peak_src == "measured"
-                else "fallback (B200_PROFILING.md)",
-                "kernel": "a3 mat-vec statement kernels of one configuration (rowdot/colsum/axpby)",
-                "algorithmic_bytes_per_launch": round(kb / max(n_kernel_groups, 1)),
-                "avg_launch_ms": round(kt / max(n_kernel_groups, 1), 5)}
-    conv_roof = {"achieved": round(cb / (ct * 1e-3) / 1e9, 1), "frac": round(cb / (ct * 1e-3) / 1e9 / hbm, 4)} \
-        if ct > 0 else None
+    ratios = {}
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            ratios = json.load(open(tp))
+        except Exception:
+            ratios = {}
+    psrc = (peak_src + " (MEASURED_PEAKS.json hbm_gbs)") if peak_src == "measured" \
+        else "fallback (B200_PROFILING.md)"
+
+    def hbm_roof(bytes_, ms_, n_, kernel, ratio_key):
+        if ms_ <= 0 or n_ == 0:
+            return None
+        ach = bytes_ / (ms_ * 1e-3) / 1e9
+        per = bytes_ / n_
+        r = ratios.get(ratio_key)
+        return {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "unit": "GB/s",
+                "frac": round(ach / hbm, 4), "traffic": round(r * per) if r else None,
+                "peak_source": psrc, "kernel": kernel,
+                "algorithmic_bytes_per_launch": round(per), "avg_launch_ms": round(ms_ / n_, 5)}
+
+    n_conv_groups = sum(1 for a in apps for r in last[a["kind"]]
+                        if convert_bytes(a["app"].objects, decode(int(r["config_id"]), a["app"].num_objects)))
+    roof_a3 = hbm_roof(kb, kt, n_kernel_groups,
+                       "a3 mat-vec statement kernels of one configuration (tile_kernel + finalizers)",
+                       "ratio")
+    roof_a2 = hbm_roof(cb, ct, n_conv_groups,
+                       "a2 conversion kernels of one configuration (convert_kernel)", "convert_ratio")
+    roof_mm = contraction_roofline(apps, last) if kb == 0 else None
+    # the dominant phase's kernel is THE roofline; the other is reported beside it
+    if roof_mm is not None:
+        roof, conv_roof = roof_mm, roof_a2
+    elif phase["convert"] > phase["kernel"] and roof_a2 is not None:
+        roof, conv_roof = roof_a2, roof_a3
+    else:
+        roof, conv_roof = roof_a3, roof_a2
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
@@ -470,7 +536,7 @@ def main():
         "e2e": e2e, "gpu_launches": launches,
         "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
         "phase_share": {k: round(v / tot_phase, 4) for k, v in phase.items()} if tot_phase else None,
-        "conversion_roofline_in_sweep": conv_roof,
+        "roofline_secondary": conv_roof,
         "conversion_gbs": conv,
         "speedup_vs_fp32_at_toq": speedup,
     }

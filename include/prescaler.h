@@ -164,6 +164,33 @@ PS_API ps_status ps_run_config(ps_app *app, const int *prec, double toq, void *s
 PS_API ps_status ps_sweep(ps_app *app, const uint64_t *config_ids, size_t n_configs, double toq,
                    void *stream, ps_result *results, int64_t *best_index);
 
+/* ------------------------------------------------------------------------- */
+/* (6) Decision-tree search (Sec. 4.4; Alg. 1 lines 1-13), with   */
+/*   ps_run_config as RunApp (Alg. 1 line 8):                                 */
+/*   - pre-full-precision scaling (Sec. 4.4.1): run the 3 uniform      */
+/*     configurations, start from the fastest passing one;                    */
+/*   - objects in descending order of their data volume (bytes x statements  */
+/*     touching them; the device-only stand-in for "the sum of the execution  */
+/*     times of related events");                                      */
+/*   - per object, normal search: targets in descending precision,    */
+/*     skipping the current type, stop at the first TOQ failure (line 10),   */
+/*     keep the fastest passing (line 12).                                    */
+/*   The wildcard test (lines 14-32) needs host-side transient conversions   */
+/*   and is not part of this device-only path.  Each trial is timed as the   */
+/*   median total_ms of `repeats` runs; a configuration is never re-run.      */
+typedef struct {
+  uint64_t config_id;     /* chosen configuration                               */
+  float total_ms;         /* its median measured time                           */
+  float pfp_ms;           /* time of the PFP starting configuration             */
+  double quality;         /* its quality                                        */
+  int32_t pass;           /* chosen configuration passes TOQ                    */
+  int32_t trials;         /* distinct configurations executed (RunApp calls)    */
+  uint64_t pfp_id;        /* PFP starting configuration                         */
+  uint64_t trial_ids[64]; /* executed configurations in order (first 64)        */
+} ps_search_result;
+PS_API ps_status ps_search(ps_app *app, double toq, int repeats, void *stream,
+                           ps_search_result *out);
+
 #ifdef __cplusplus
 }
 #endif

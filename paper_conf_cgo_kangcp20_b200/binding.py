@@ -28,7 +28,7 @@ SYMBOLS = [
     "ps_app_create", "ps_app_destroy", "ps_app_num_objects", "ps_app_object_info",
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
-    "ps_run_config", "ps_sweep",
+    "ps_run_config", "ps_sweep", "ps_search",
 ]
 
 
@@ -55,6 +55,13 @@ class PsResult(ctypes.Structure):
                 ("reserved", ctypes.c_float), ("quality", ctypes.c_double),
                 ("max_rel", ctypes.c_double), ("nonfinite", ctypes.c_uint64),
                 ("pass_", ctypes.c_int32), ("status", ctypes.c_int32)]
+
+
+class PsSearchResult(ctypes.Structure):
+    _fields_ = [("config_id", ctypes.c_uint64), ("total_ms", ctypes.c_float),
+                ("pfp_ms", ctypes.c_float), ("quality", ctypes.c_double), ("pass_", ctypes.c_int32),
+                ("trials", ctypes.c_int32), ("pfp_id", ctypes.c_uint64),
+                ("trial_ids", ctypes.c_uint64 * 64)]
 
 
 RESULT_DTYPE = np.dtype([("config_id", "<u8"), ("convert_ms", "<f4"), ("kernel_ms", "<f4"),
@@ -104,6 +111,8 @@ def lib():
                                                  ctypes.POINTER(PsResult)]),
                 "ps_sweep": (ctypes.c_int, [vp, ctypes.POINTER(ctypes.c_uint64), ctypes.c_size_t,
                                             ctypes.c_double, vp, ctypes.POINTER(PsResult), i64p]),
+                "ps_search": (ctypes.c_int, [vp, ctypes.c_double, ctypes.c_int, vp,
+                                             ctypes.POINTER(PsSearchResult)]),
             }
             for name, (res, args) in sig.items():
                 f = getattr(L, name)
@@ -285,6 +294,16 @@ class App:
                "ps_sweep")
         arr = np.frombuffer(bytes(res), dtype=RESULT_DTYPE)[:len(ids)].copy()
         return arr, int(best.value)
+
+    def search(self, toq: float = 0.9, repeats: int = 1, stream=None) -> dict:
+        """ps_search: PFP initialisation + Alg. 1 normal search (decision tree)."""
+        r = PsSearchResult()
+        _check(lib().ps_search(self._h, float(toq), int(repeats), _stream(stream), ctypes.byref(r)),
+               "ps_search")
+        return {"config_id": int(r.config_id), "prec": self.decode(r.config_id),
+                "total_ms": float(r.total_ms), "quality": float(r.quality), "pass": bool(r.pass_),
+                "trials": int(r.trials), "pfp_id": int(r.pfp_id), "pfp_ms": float(r.pfp_ms),
+                "trial_ids": [int(x) for x in r.trial_ids[:min(r.trials, 64)]]}
 
     def sweep(self, config_ids, toq: float = 0.9, stream=None):
         arr, best = self.sweep_raw(config_ids, toq, stream)

@@ -19,6 +19,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <map>
 #include <vector>
 
 #include "common.cuh"
@@ -78,6 +79,17 @@ static const AppDef kApps[] = {
     {"covar", 3, 2, {{"data", 2, 0}, {"mean", 3, 0}, {"symmat", 1, 1}}},
 };
 enum AppKind { K_GEMM, K_2MM, K_3MM, K_ATAX, K_BICG, K_GESUMMV, K_CORR, K_COVAR };
+// statements that read or write each object (for ps_search's object order)
+static const int kTouch[8][8] = {
+    {1, 1, 1},                  // gemm: C <- aAB + bC
+    {1, 1, 2, 1, 1},            // 2mm
+    {1, 1, 1, 1, 2, 2, 1},      // 3mm
+    {2, 1, 1, 2},               // atax
+    {2, 1, 1, 1, 1},            // bicg
+    {1, 1, 2, 2, 2},            // gesummv
+    {4, 3, 2, 1},               // corr
+    {3, 2, 1},                  // covar
+};
 
 }  // namespace ps
 
@@ -597,6 +609,108 @@ ps_status ps_sweep(ps_app *a, const uint64_t *ids, size_t n, double toq, void *s
         (results[i].total_ms == results[*best].total_ms && results[i].config_id < results[*best].config_id))
       *best = (int64_t)i;
   }
+  return PS_OK;
+}
+
+// Decision-tree search (Sec. 4.4, Alg. 1 normal search + Sec. 4.4.1 PFP), see prescaler.h.
+ps_status ps_search(ps_app *a, double toq, int repeats, void *stream, ps_search_result *out) {
+  ps_status s = ready(a);
+  if (s != PS_OK) return s;
+  if (!out || repeats < 1) { set_error("ps_search: bad argument"); return PS_ERR_INVALID; }
+  memset(out, 0, sizeof(*out));
+  const int M = a->def->nobj;
+  struct Trial { float ms; double q; bool pass; };
+  std::map<uint64_t, Trial> seen;
+  auto encode = [&](const int *prec) {
+    uint64_t id = 0, w = 1;
+    for (int m = 0; m < M; m++) { id += (uint64_t)prec[m] * w; w *= 3; }
+    return id;
+  };
+  // RunApp (Alg. 1 line 8): median total time of `repeats` runs; never re-run a config
+  auto run = [&](const int *prec, Trial *t) -> ps_status {
+    const uint64_t id = encode(prec);
+    auto it = seen.find(id);
+    if (it != seen.end()) { *t = it->second; return PS_OK; }
+    std::vector<float> ms;
+    ps_result r{};
+    for (int k = 0; k < repeats; k++) {
+      ps_status e = ps_run_config(a, prec, toq, stream, &r);
+      if (e != PS_OK) return e;
+      ms.push_back(r.total_ms);
+    }
+    std::sort(ms.begin(), ms.end());
+    *t = Trial{ms[ms.size() / 2], r.quality, r.pass != 0};
+    seen[id] = *t;
+    if (out->trials < 64) out->trial_ids[out->trials] = id;
+    out->trials++;
+    return PS_OK;
+  };
+  auto better = [](const Trial &x, uint64_t xi, const Trial &y, uint64_t yi) {
+    return x.ms < y.ms || (x.ms == y.ms && xi < yi);
+  };
+
+  // Sec. 4.4.1 pre-full-precision scaling: uniform configurations, descending precision
+  int cur[8], cand[8];
+  Trial tcur{0.f, 0.0, false};
+  bool have = false;
+  uint64_t cur_id = 0;
+  for (int t = PS_F64; t <= PS_F16; t++) {
+    for (int m = 0; m < M; m++) cand[m] = t;
+    Trial tr;
+    if ((s = run(cand, &tr)) != PS_OK) return s;
+    const uint64_t id = encode(cand);
+    if (tr.pass && (!have || better(tr, id, tcur, cur_id))) {
+      memcpy(cur, cand, sizeof(cand));
+      tcur = tr;
+      cur_id = id;
+      have = true;
+    }
+  }
+  if (!have) {   // no uniform configuration passes: start from the full-precision one
+    for (int m = 0; m < M; m++) cur[m] = PS_F64;
+    cur_id = 0;
+    if ((s = run(cur, &tcur)) != PS_OK) return s;
+  }
+  out->pfp_id = cur_id;
+  out->pfp_ms = tcur.ms;
+
+  // objects in descending order of data volume, ties -> lower index
+  int order[8];
+  for (int m = 0; m < M; m++) order[m] = m;
+  std::stable_sort(order, order + M, [&](int x, int y) {
+    const double wx = (double)nelem(a, x) * kTouch[a->kind][x];
+    const double wy = (double)nelem(a, y) * kTouch[a->kind][y];
+    return wx > wy;
+  });
+  // Alg. 1 lines 1-13 per object
+  for (int oi = 0; oi < M; oi++) {
+    const int m = order[oi];
+    int best[8];
+    memcpy(best, cur, sizeof(cur));
+    Trial tbest = tcur;
+    uint64_t best_id = cur_id;
+    for (int t = PS_F64; t <= PS_F16; t++) {          // descending precision
+      if (t == cur[m]) continue;                       // line 3
+      memcpy(cand, cur, sizeof(cur));
+      cand[m] = t;
+      Trial tr;
+      if ((s = run(cand, &tr)) != PS_OK) return s;     // line 8
+      if (!tr.pass) break;                             // line 10: stop at the first failure
+      const uint64_t id = encode(cand);
+      if (better(tr, id, tbest, best_id)) {            // line 12
+        memcpy(best, cand, sizeof(cand));
+        tbest = tr;
+        best_id = id;
+      }
+    }
+    memcpy(cur, best, sizeof(best));
+    tcur = tbest;
+    cur_id = best_id;
+  }
+  out->config_id = cur_id;
+  out->total_ms = tcur.ms;
+  out->quality = tcur.q;
+  out->pass = tcur.pass;
   return PS_OK;
 }
 
