@@ -243,6 +243,234 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   }
 }
 
+// ===================================================================
+// 2-CTA persistent variant: a cluster of 2 CTAs (one TPC) computes a 256 x 256
+// tile with tcgen05.mma.cta_group::2 (M=256, N=256, K=16).  Each CTA stages
+// 128 rows of A and 128 columns of B per k-block (32 KiB / stage, 6 stages);
+// TMA in both CTAs completes on the leader's full barrier; the leader's single
+// MMA thread commits (multicast) to both CTAs' empty / tmem_full barriers.
+// Two TMEM accumulators (2 x 256 columns) let the epilogue of tile i overlap
+// the MMAs of tile i+1.  Tiles are walked persistently, cluster c taking tiles
+// c, c + #clusters, ... (SYRK: lower tiles skipped by every role alike).
+namespace tc2 {
+
+constexpr int BM = 256, BN = 256, BK = 64, STAGES = 6;
+constexpr int HM = BM / 2, HN = BN / 2;          // per-CTA halves
+constexpr int A_BYTES = HM * BK * 2;            // 16 KiB
+constexpr int B_BYTES = HN * BK * 2;            // 16 KiB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512;
+constexpr int NTHREADS = 192;
+constexpr uint32_t TMEM_COLS = 512;             // 2 accumulators x 256 f32 columns
+constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;     // shared::cluster address of the leader's copy
+
+using tc::Params;
+using tc::fence_after;
+using tc::fence_before;
+using tc::mbar_expect_tx;
+using tc::mbar_init;
+using tc::mbar_wait;
+using tc::smem_u32;
+using tc::tmem_ld16;
+using tc::umma_desc;
+using tc::load_c;
+using tc::store_c;
+
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tma_load_2sm(void *dst, const CUtensorMap *map, uint64_t *bar, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, "
+      "%4}], [%2];" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)map), "r"(smem_u32(bar) & PEER_MASK), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void umma2(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  const uint32_t z = 0;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, {%5, %5, %5, %5, %5, %5, %5, %5}, p;\n\t}" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(z));
+}
+__device__ __forceinline__ void commit_both(uint64_t *bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          smem_u32(bar)),
+      "h"((uint16_t)3)
+      : "memory");
+}
+// arrive on the leader CTA's copy of a barrier (remote for rank 1)
+__device__ __forceinline__ void arrive_leader(uint64_t *bar) {
+  uint32_t remote;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(remote) : "r"(smem_u32(bar)));
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(remote) : "memory");
+}
+
+struct Sched {
+  int64_t tiles_m, tiles_n, total;
+  int upper_only;
+  // i-th tile of this cluster (skipping SYRK lower tiles); false when exhausted
+  __device__ bool get(int64_t cluster, int64_t nclusters, int64_t &cursor, int &m0, int &n0) const {
+    for (int64_t t = cursor; t < total; t += nclusters) {
+      const int64_t tm = t / tiles_n, tn = t % tiles_n;
+      if (upper_only && tm > tn) continue;
+      m0 = (int)(tm * BM);
+      n0 = (int)(tn * BN);
+      cursor = t + nclusters;
+      return true;
+    }
+    cursor = total;
+    return false;
+  }
+};
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
+    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
+                    Params p, Sched sch) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t *sA = smem;
+  uint8_t *sB = smem + STAGES * A_BYTES;
+  uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
+  uint64_t *empty = full + STAGES;
+  uint64_t *tfull = empty + STAGES;      // [2]
+  uint64_t *tempty = tfull + 2;          // [2]
+  uint32_t *tmem_slot = (uint32_t *)(tempty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const bool leader = rank == 0;
+  const int64_t cluster = blockIdx.x >> 1, nclusters = gridDim.x >> 1;
+  const int nk = (p.K + BK - 1) / BK;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tma_a) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tma_b) : "memory");
+    for (int s = 0; s < STAGES; s++) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; a++) {
+      mbar_init(&tfull[a], 1);
+      mbar_init(&tempty[a], 8);          // 4 epilogue warps x 2 CTAs
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {   // same warp in both CTAs (cta_group::2 allocation)
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  fence_before();
+  cluster_sync_all();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {   // ---------------- TMA producer (both CTAs)
+      int64_t cursor = cluster;
+      int m0, n0;
+      uint32_t it = 0;
+      while (sch.get(cluster, nclusters, cursor, m0, n0)) {
+        const int am = m0 + (int)rank * HM, bn = n0 + (int)rank * HN;
+        for (int kb = 0; kb < nk; kb++, it++) {
+          const int s = it % STAGES;
+          const uint32_t ph = (it / STAGES) & 1u;
+          mbar_wait(&empty[s], ph ^ 1u);
+          if (leader) mbar_expect_tx(&full[s], 2 * STAGE_BYTES);   // both CTAs' bytes
+          const int k0 = kb * BK;
+          uint8_t *a = sA + s * A_BYTES;
+          if (!p.a_mn_major) {
+            tma_load_2sm(a, &tma_a, &full[s], k0, am);                    // box {64 K, 128 M}
+          } else {
+            tma_load_2sm(a, &tma_a, &full[s], am, k0);                    // box {64 M, 64 K} x 2
+            tma_load_2sm(a + tc::BOX_BYTES, &tma_a, &full[s], am + 64, k0);
+          }
+          uint8_t *b = sB + s * B_BYTES;
+          tma_load_2sm(b, &tma_b, &full[s], bn, k0);                      // box {64 N, 64 K} x 2
+          tma_load_2sm(b + tc::BOX_BYTES, &tma_b, &full[s], bn + 64, k0);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (leader && lane == 0) {   // ---- MMA issuer (leader CTA, single thread)
+      const uint32_t idesc = (1u << 4) | ((uint32_t)p.a_mn_major << 15) | (1u << 16) |
+                             ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+      int64_t cursor = cluster;
+      int m0, n0;
+      uint32_t it = 0, j = 0;
+      while (sch.get(cluster, nclusters, cursor, m0, n0)) {
+        const uint32_t acc = j & 1u;
+        mbar_wait(&tempty[acc], ((j >> 1) & 1u) ^ 1u);   // epilogues of both CTAs drained it
+        fence_after();
+        const uint32_t dcol = tmem + acc * BN;
+        for (int kb = 0; kb < nk; kb++, it++) {
+          const int s = it % STAGES;
+          mbar_wait(&full[s], (it / STAGES) & 1u);
+          fence_after();
+          const uint32_t abase = smem_u32(sA + s * A_BYTES), bbase = smem_u32(sB + s * B_BYTES);
+#pragma unroll
+          for (int kk = 0; kk < BK / 16; kk++) {
+            const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * 2048, tc::BOX_BYTES, 1024)
+                                             : umma_desc(abase + kk * 32, 16, 1024);
+            const uint64_t bd = umma_desc(bbase + kk * 2048, tc::BOX_BYTES, 1024);
+            umma2(dcol, ad, bd, idesc, (kb | kk) != 0);
+          }
+          commit_both(&empty[s]);   // stage s free in both CTAs once these MMAs retire
+        }
+        commit_both(&tfull[acc]);   // accumulator acc complete in both CTAs
+        j++;
+      }
+    }
+  } else {   // ------------------------- epilogue warps 2..5 (both CTAs)
+    const int q = warp & 3;
+    int64_t cursor = cluster;
+    int m0, n0;
+    uint32_t j = 0;
+    while (sch.get(cluster, nclusters, cursor, m0, n0)) {
+      const uint32_t acc = j & 1u;
+      mbar_wait(&tfull[acc], (j >> 1) & 1u);
+      fence_after();
+      const int64_t row = (int64_t)m0 + rank * HM + q * 32 + lane;
+      for (int cc = 0; cc < BN / 16; cc++) {
+        uint32_t v[16];
+        tmem_ld16(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * 16), v);
+        if (row < p.M) {
+#pragma unroll
+          for (int e = 0; e < 16; e++) {
+            const int64_t col = (int64_t)n0 + cc * 16 + e;
+            if (col >= p.N) break;
+            float r = __uint_as_float(v[e]);
+            const int64_t idx = row * p.ldc + col;
+            if (p.epi == EPI_AXPBY) r = __fmaf_rn(p.alpha, r, p.beta * load_c(p.Cin, p.cin_type, idx));
+            else if (p.epi == EPI_DIV) r = r / p.div;
+            store_c(p.C, p.c_type, idx, r);
+          }
+        }
+      }
+      fence_before();
+      __syncwarp();
+      if (lane == 0) arrive_leader(&tempty[acc]);
+      j++;
+    }
+  }
+  fence_before();
+  __syncthreads();
+  cluster_sync_all();   // both CTAs finished with TMEM and with each other's barriers
+  if (warp == 1) {
+    fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS));
+  }
+}
+
+}  // namespace tc2
 }  // namespace tc
 
 // ------------------------------------------------------------------ host
@@ -305,6 +533,29 @@ ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
   }
   Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
            (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only};
+  if ((g.M > BM || g.N > BN) && !getenv("PS_TC_1SM")) {   // 2-CTA persistent path
+    using namespace tc2;
+    static bool attr2 = false;
+    if (!attr2) {
+      PS_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   tc2::SMEM_BYTES));
+      attr2 = true;
+    }
+    Sched sch;
+    sch.tiles_m = (g.M + tc2::BM - 1) / tc2::BM;
+    sch.tiles_n = (g.N + tc2::BN - 1) / tc2::BN;
+    sch.total = sch.tiles_m * sch.tiles_n;
+    sch.upper_only = g.upper_only;
+    int64_t work = 0;
+    for (int64_t t = 0; t < sch.total; t++)
+      if (!g.upper_only || t / sch.tiles_n <= t % sch.tiles_n) work++;
+    int64_t clusters = num_sms() / 2;
+    if (clusters > work) clusters = work;
+    if (clusters < 1) clusters = 1;
+    gemm_tc2_kernel<<<(unsigned)(2 * clusters), tc2::NTHREADS, tc2::SMEM_BYTES, st>>>(ma, mb, p, sch);
+    PS_CHECK_LAUNCH("gemm_tc2_kernel");
+    return PS_OK;
+  }
   dim3 grid((unsigned)((g.N + BN - 1) / BN), (unsigned)((g.M + BM - 1) / BM));
   gemm_tc_kernel<<<grid, NTHREADS, SMEM_BYTES, st>>>(ma, mb, p);
   PS_CHECK_LAUNCH("gemm_tc_kernel");
