@@ -1,0 +1,31 @@
+"""compute-sanitizer over small shapes of every kernel family (SURVEY §4 tier 4)."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer(tool):
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(cs):
+        pytest.skip("compute-sanitizer not found")
+    from paper_conf_cgo_kangcp20_b200 import build
+    build.build()
+    env = dict(os.environ)
+    if tool == "racecheck":
+        # tcgen05.alloc.cta_group::2 writes the same TMEM address into the same smem
+        # slot of BOTH CTAs of the pair (the 2-SM allocation idiom, identical values);
+        # racecheck reports that as a write/write race.  Race-check the shared-memory
+        # protocol on the 1-SM tensor path; memcheck / synccheck cover the 2-CTA path.
+        env["PS_TC_1SM"] = "1"
+    r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "17", sys.executable,
+                        os.path.join(ROOT, "tools", "sanitize_run.py")],
+                       capture_output=True, text=True, timeout=1500, env=env)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0 and "sanitize run ok" in r.stdout, tail
