@@ -141,8 +141,8 @@ typedef struct {
   float kernel_ms;    /* a3: precision-scaled kernels                          */
   float backconv_ms;  /* a4+a5 fused: back-conversion + per-element error      */
   float quality_ms;   /* a5: final deterministic reduction                     */
-  float total_ms;     /* convert + kernel + backconv  (reading #19)            */
-  float reserved;
+  float total_ms;     /* [transfer +] convert + kernel + backconv  (reading #19) */
+  float transfer_ms;  /* host conversion + H2D + D2H (ps_run_config_host only)  */
   double quality;     /* 1 - mean relative error                               */
   double max_rel;     /* max uncapped relative error                           */
   uint64_t nonfinite; /* non-finite delivered output elements                  */
@@ -163,6 +163,39 @@ PS_API ps_status ps_run_config(ps_app *app, const int *prec, double toq, void *s
 /* lowest id), -1 if none passes.  One stream synchronisation at the end.      */
 PS_API ps_status ps_sweep(ps_app *app, const uint64_t *config_ids, size_t n_configs, double toq,
                    void *stream, ps_result *results, int64_t *best_index);
+
+/* ------------------------------------------------------------------------- */
+/* (5b) Whole-program evaluation with host<->device transfers ("the  */
+/*   input data of target kernels are translated to a lower precision before */
+/*   data transfer from the host").  Per input object a type-conversion method */
+/*   (Fig. 3):                                                     */
+/*     PS_XFER_DEVICE      (c) H2D at orig (f32), device-side conversion      */
+/*     PS_XFER_HOST_LOOP   (a) host single-loop (scalar) conversion, H2D at c(m) */
+/*     PS_XFER_HOST_SIMD   (b) host multithreaded SIMD conversion, H2D at c(m) */
+/*     PS_XFER_PIPELINE    (e) (b) in 16 MiB chunks overlapped with their H2D   */
+/*     PS_XFER_TRANSIENT   (d) host -> fp16 (the intermediate type), H2D fp16, */
+/*                             device fp16 -> c(m) (can add error)      */
+typedef enum {
+  PS_XFER_DEVICE = 0,
+  PS_XFER_HOST_LOOP = 1,
+  PS_XFER_HOST_SIMD = 2,
+  PS_XFER_PIPELINE = 3,
+  PS_XFER_TRANSIENT = 4
+} ps_xfer_method;
+/* Host-side RNE conversion of an f32 array (canonical NaN, bit-identical to   */
+/* ps_convert): dst_type f64/f32/f16, `threads` workers (<= 1: caller's),     */
+/* simd != 0 uses F16C/AVX2 when the CPU has them.  Host pointers.            */
+PS_API ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, int threads,
+                                 int simd);
+/* Evaluate one configuration from HOST f32 inputs (host_inputs[m] for role   */
+/* in/inout, pinned memory recommended): per-object method `methods[m]`      */
+/* (NULL = all PS_XFER_DEVICE), `threads` host workers; the delivered f32     */
+/* outputs are read back into host_outputs[m] when non-NULL.  Synchronous;    */
+/* out->transfer_ms = host conversion + transfers (wall clock), and          */
+/* out->total_ms includes it.                                                 */
+PS_API ps_status ps_run_config_host(ps_app *app, const int *prec, const int *methods,
+                                    const void *const *host_inputs, void *const *host_outputs,
+                                    int threads, double toq, void *stream, ps_result *out);
 
 /* ------------------------------------------------------------------------- */
 /* (6) Decision-tree search (Sec. 4.4; Alg. 1 lines 1-13), with   */

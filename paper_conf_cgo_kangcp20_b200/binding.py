@@ -28,8 +28,10 @@ SYMBOLS = [
     "ps_app_create", "ps_app_destroy", "ps_app_num_objects", "ps_app_object_info",
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
-    "ps_run_config", "ps_sweep", "ps_search",
+    "ps_run_config", "ps_sweep", "ps_search", "ps_host_convert", "ps_run_config_host",
 ]
+# type-conversion methods for host inputs (Fig. 3)
+XFER_DEVICE, XFER_HOST_LOOP, XFER_HOST_SIMD, XFER_PIPELINE, XFER_TRANSIENT = 0, 1, 2, 3, 4
 
 
 class PsError(RuntimeError):
@@ -52,7 +54,7 @@ class PsResult(ctypes.Structure):
     _fields_ = [("config_id", ctypes.c_uint64), ("convert_ms", ctypes.c_float),
                 ("kernel_ms", ctypes.c_float), ("backconv_ms", ctypes.c_float),
                 ("quality_ms", ctypes.c_float), ("total_ms", ctypes.c_float),
-                ("reserved", ctypes.c_float), ("quality", ctypes.c_double),
+                ("transfer_ms", ctypes.c_float), ("quality", ctypes.c_double),
                 ("max_rel", ctypes.c_double), ("nonfinite", ctypes.c_uint64),
                 ("pass_", ctypes.c_int32), ("status", ctypes.c_int32)]
 
@@ -66,7 +68,7 @@ class PsSearchResult(ctypes.Structure):
 
 RESULT_DTYPE = np.dtype([("config_id", "<u8"), ("convert_ms", "<f4"), ("kernel_ms", "<f4"),
                          ("backconv_ms", "<f4"), ("quality_ms", "<f4"), ("total_ms", "<f4"),
-                         ("reserved", "<f4"), ("quality", "<f8"), ("max_rel", "<f8"),
+                         ("transfer_ms", "<f4"), ("quality", "<f8"), ("max_rel", "<f8"),
                          ("nonfinite", "<u8"), ("pass", "<i4"), ("status", "<i4")])
 assert ctypes.sizeof(PsResult) == 64 and RESULT_DTYPE.itemsize == 64
 
@@ -113,6 +115,12 @@ def lib():
                                             ctypes.c_double, vp, ctypes.POINTER(PsResult), i64p]),
                 "ps_search": (ctypes.c_int, [vp, ctypes.c_double, ctypes.c_int, vp,
                                              ctypes.POINTER(PsSearchResult)]),
+                "ps_host_convert": (ctypes.c_int, [vp, vp, ctypes.c_int, ctypes.c_size_t, ctypes.c_int,
+                                                   ctypes.c_int]),
+                "ps_run_config_host": (ctypes.c_int, [vp, ctypes.POINTER(ctypes.c_int),
+                                                      ctypes.POINTER(ctypes.c_int), ctypes.POINTER(vp),
+                                                      ctypes.POINTER(vp), ctypes.c_int, ctypes.c_double,
+                                                      vp, ctypes.POINTER(PsResult)]),
             }
             for name, (res, args) in sig.items():
                 f = getattr(L, name)
@@ -171,6 +179,16 @@ def ps_convert(src, src_type: int, dst, dst_type: int, n: int = None, stream=Non
         n = src.numel()
     _check(lib().ps_convert(_ptr(src), src_type, _ptr(dst), dst_type, n, _stream(stream)),
            "ps_convert")
+
+
+def ps_host_convert(src: np.ndarray, dst_type: int, threads: int = 0, simd: bool = True) -> np.ndarray:
+    """Host-side RNE conversion of an f32 numpy array (Fig. 3a: simd=False, threads=1;
+    Fig. 3b: SIMD + threads).  Bit-identical to ps_convert."""
+    src = np.ascontiguousarray(src, dtype=np.float32)
+    out = np.empty(src.shape, dtype={F64: np.float64, F32: np.float32, F16: np.float16}[dst_type])
+    _check(lib().ps_host_convert(src.ctypes.data, out.ctypes.data, dst_type, src.size, threads,
+                                 1 if simd else 0), "ps_host_convert")
+    return out
 
 
 # -------------------------------------------------------------- (2) quality
@@ -294,6 +312,21 @@ class App:
                "ps_sweep")
         arr = np.frombuffer(bytes(res), dtype=RESULT_DTYPE)[:len(ids)].copy()
         return arr, int(best.value)
+
+    def run_config_host(self, prec, host_inputs, methods=None, host_outputs=None, threads: int = 0,
+                        toq: float = 0.9, stream=None) -> dict:
+        """ps_run_config_host: the configuration from host f32 inputs with per-object
+        conversion methods (XFER_*); transfer_ms and total_ms include the transfers."""
+        m = self.num_objects
+        p = (ctypes.c_int * m)(*prec)
+        meth = None if methods is None else (ctypes.c_int * m)(*methods)
+        hin = (vp * m)(*[_ptr(t) if t is not None else None for t in host_inputs])
+        hout = None if host_outputs is None else (vp * m)(*[_ptr(t) if t is not None else None
+                                                          for t in host_outputs])
+        r = PsResult()
+        _check(lib().ps_run_config_host(self._h, p, meth, hin, hout, int(threads), float(toq),
+                                        _stream(stream), ctypes.byref(r)), "ps_run_config_host")
+        return _result_dict(np.frombuffer(bytes(r), dtype=RESULT_DTYPE)[0])
 
     def search(self, toq: float = 0.9, repeats: int = 1, stream=None) -> dict:
         """ps_search: PFP initialisation + Alg. 1 normal search (decision tree)."""

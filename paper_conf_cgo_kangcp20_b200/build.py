@@ -4,7 +4,9 @@
 csrc/ is compiled separately (in parallel) with
 ``-gencode arch=compute_100a,code=sm_100a -lineinfo -O3 -fmad=false`` (no FMA
 contraction: every fused multiply-add in the kernels is written explicitly,
-readings R3/R4) and linked with the static CUDA runtime.
+readings R3/R4); the host-only .cpp sources (host-side conversion, Fig. 3a/3b)
+with g++ -O3 (SIMD paths selected at run time by CPU feature checks).  Linked
+with the static CUDA runtime.
 """
 from __future__ import annotations
 
@@ -20,13 +22,16 @@ INCLUDE = os.path.join(os.path.dirname(HERE), "include")
 LIB = os.path.join(HERE, "libprescaler.so")
 OBJDIR = os.path.join(HERE, "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+CXX = os.environ.get("CXX", "g++")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-fmad=false", "-Xcompiler", "-fPIC",
          "-Xcompiler", "-fvisibility=hidden", "-I" + INCLUDE, "--expt-relaxed-constexpr"]
+CXXFLAGS = ["-O3", "-std=c++17", "-fPIC", "-fvisibility=hidden", "-ffp-contract=off", "-pthread",
+            "-I" + INCLUDE]
 
 
 def _sources():
-    return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
 
 
 def _deps():
@@ -45,12 +50,15 @@ def _compile(src, verbose):
     hdrs = glob.glob(os.path.join(CSRC, "*.cuh")) + [os.path.join(INCLUDE, "prescaler.h")]
     if not _stale(obj, [src] + hdrs):
         return obj
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
+    if src.endswith(".cpp"):
+        cmd = [CXX, *CXXFLAGS, "-c", src, "-o", obj]
+    else:
+        cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
+        if verbose:
+            cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
-        raise RuntimeError("nvcc failed for %s:\n%s%s" % (src, r.stdout, r.stderr))
+        raise RuntimeError("compile failed for %s:\n%s%s" % (src, r.stdout, r.stderr))
     if verbose and r.stderr:
         sys.stderr.write(r.stderr)
     return obj
@@ -66,7 +74,7 @@ def build(force: bool = False, verbose: bool = False, jobs: int = 8) -> str:
     with cf.ThreadPoolExecutor(jobs) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), _sources()))
     tmp = LIB + ".tmp%d" % os.getpid()
-    cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs]
+    cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-Xcompiler", "-pthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("link failed:\n" + r.stdout + r.stderr)

@@ -19,7 +19,9 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <map>
+#include <thread>
 #include <vector>
 
 #include "common.cuh"
@@ -115,6 +117,15 @@ struct ps_app {
   // workspace layout
   size_t slot_off[8] = {0};
   size_t partial_off = 0, qparts_off = 0, qres_off = 0, total = 0;
+  size_t trans_off[8] = {0};
+  // host-transfer path (ps_run_config_host): per input object, where a2 takes
+  // its data from: 0 = orig_in (device conversion), 1 = already in the slot at
+  // c(m) (host conversion + H2D), 2 = fp16 intermediate in the transient region
+  int pre[8] = {0};
+  void *pinned = nullptr;          // host staging (largest converted input)
+  size_t pinned_bytes = 0;
+  void *ring[2] = {nullptr, nullptr};
+  cudaEvent_t ring_ev[2] = {nullptr, nullptr};
   // timing
   std::vector<cudaEvent_t> ev;
   QPart *host_res = nullptr;   // pinned, MAX_BATCH
@@ -122,6 +133,11 @@ struct ps_app {
   ~ps_app() {
     for (auto e : ev) cudaEventDestroy(e);
     if (host_res) cudaFreeHost(host_res);
+    if (pinned) cudaFreeHost(pinned);
+    for (int k = 0; k < 2; k++) {
+      if (ring[k]) cudaFreeHost(ring[k]);
+      if (ring_ev[k]) cudaEventDestroy(ring_ev[k]);
+    }
   }
 };
 
@@ -175,6 +191,10 @@ void layout(ps_app *a) {
   off = align_up(off + (size_t)nout * QBLOCKS_MAX * sizeof(QPart), 256);
   a->qres_off = off;
   off = align_up(off + (size_t)MAX_BATCH * sizeof(QPart), 256);
+  for (int m = 0; m < a->def->nobj; m++) {   // transient (fp16 intermediate) region per input
+    a->trans_off[m] = off;
+    if (a->def->o[m].role == 0 || a->def->o[m].role == 2) off = align_up(off + nelem(a, m) * 2, 256);
+  }
   a->total = off;
 }
 
@@ -323,7 +343,12 @@ ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res
     c.ptr[m] = a->ws + a->slot_off[m];
     const int role = a->def->o[m].role;
     if (role == 0 || role == 2) {
-      if (role == 0 && prec[m] == PS_F32) {
+      if (a->pre[m] == 1) {
+        // host-converted and transferred at c(m) already (ps_run_config_host)
+      } else if (a->pre[m] == 2) {   // transient: fp16 intermediate -> c(m) on the device
+        ps_status s = convert_async(a->ws + a->trans_off[m], PS_F16, c.ptr[m], prec[m], nelem(a, m), st);
+        if (s != PS_OK) return s;
+      } else if (role == 0 && prec[m] == PS_F32) {
         c.ptr[m] = (void *)a->orig_in[m];   // original precision: used in place
       } else {
         ps_status s = convert_async(a->orig_in[m], PS_F32, c.ptr[m], prec[m], nelem(a, m), st);
@@ -609,6 +634,115 @@ ps_status ps_sweep(ps_app *a, const uint64_t *ids, size_t n, double toq, void *s
         (results[i].total_ms == results[*best].total_ms && results[i].config_id < results[*best].config_id))
       *best = (int64_t)i;
   }
+  return PS_OK;
+}
+
+ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, int threads, int simd) {
+  if (!dtype_ok(dst_type)) { set_error("ps_host_convert: bad dtype"); return PS_ERR_INVALID; }
+  if (n && (!src || !dst)) { set_error("ps_host_convert: null pointer"); return PS_ERR_INVALID; }
+  ps::host_convert_f32(src, dst, dst_type, n, threads, simd != 0);
+  return PS_OK;
+}
+
+// Whole-program evaluation from host inputs with per-object conversion methods
+// (Fig. 3 a-e); see prescaler.h.
+ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
+                             const void *const *host_inputs, void *const *host_outputs, int threads,
+                             double toq, void *stream, ps_result *out) {
+  ps_status s = ready(a);
+  if (s != PS_OK) return s;
+  if ((s = check_prec(a, prec)) != PS_OK) return s;
+  if (!host_inputs || !out) { set_error("ps_run_config_host: null pointer"); return PS_ERR_INVALID; }
+  if ((s = ensure_events(a, NEV)) != PS_OK) return s;
+  if (threads <= 0) threads = (int)std::max(1u, std::thread::hardware_concurrency());
+  cudaStream_t st = (cudaStream_t)stream;
+  const int M = a->def->nobj;
+  constexpr size_t CH = (size_t)4 << 20;   // pipeline chunk: 4 Mi elements (16 MiB of f32)
+  // staging buffers (pinned, library-owned, grown on demand)
+  size_t need = 0;
+  for (int m = 0; m < M; m++) {
+    const int role = a->def->o[m].role;
+    if (role != 0 && role != 2) continue;
+    const int meth = methods ? methods[m] : PS_XFER_DEVICE;
+    if (meth < PS_XFER_DEVICE || meth > PS_XFER_TRANSIENT || !host_inputs[m]) {
+      set_error("ps_run_config_host: bad method or missing host input %d", m);
+      return PS_ERR_INVALID;
+    }
+    if (meth == PS_XFER_HOST_LOOP || meth == PS_XFER_HOST_SIMD) need = std::max(need, nelem(a, m) * dtype_size(prec[m]));
+    if (meth == PS_XFER_TRANSIENT) need = std::max(need, nelem(a, m) * 2);
+  }
+  if (need > a->pinned_bytes) {
+    if (a->pinned) cudaFreeHost(a->pinned);
+    a->pinned = nullptr;
+    a->pinned_bytes = 0;
+    PS_CUDA(cudaMallocHost(&a->pinned, need));
+    a->pinned_bytes = need;
+  }
+  if (!a->ring[0]) {
+    for (int k = 0; k < 2; k++) {
+      PS_CUDA(cudaMallocHost(&a->ring[k], CH * 8));
+      PS_CUDA(cudaEventCreateWithFlags(&a->ring_ev[k], cudaEventDisableTiming));
+    }
+  }
+  // ---- inputs: host conversion + H2D per object, in object order (wall clock)
+  const auto t0 = std::chrono::steady_clock::now();
+  for (int m = 0; m < M; m++) {
+    const int role = a->def->o[m].role;
+    a->pre[m] = 0;
+    if (role != 0 && role != 2) continue;
+    const int meth = methods ? methods[m] : PS_XFER_DEVICE;
+    const size_t n = nelem(a, m), es = dtype_size(prec[m]);
+    const float *src = (const float *)host_inputs[m];
+    char *slot = a->ws + a->slot_off[m];
+    if (meth == PS_XFER_DEVICE || (prec[m] == PS_F32 && role == 0 && meth != PS_XFER_TRANSIENT)) {
+      // (c): H2D at orig, the device converts in a2 (f32 inputs are used in place)
+      PS_CUDA(cudaMemcpyAsync((void *)a->orig_in[m], src, n * 4, cudaMemcpyHostToDevice, st));
+    } else if (meth == PS_XFER_TRANSIENT) {   // (d): host -> fp16, H2D fp16, device fp16 -> c(m)
+      ps::host_convert_f32(src, a->pinned, PS_F16, n, threads, true);
+      PS_CUDA(cudaMemcpyAsync(a->ws + a->trans_off[m], a->pinned, n * 2, cudaMemcpyHostToDevice, st));
+      PS_CUDA(cudaStreamSynchronize(st));
+      a->pre[m] = 2;
+    } else if (meth == PS_XFER_PIPELINE) {    // (e): chunked conversion overlapped with H2D
+      for (size_t c0 = 0, k = 0; c0 < n; c0 += CH, k++) {
+        const int b = (int)(k & 1);
+        const size_t len = std::min(CH, n - c0);
+        // the slot's previous copy (this or an earlier object) must have left the buffer
+        PS_CUDA(cudaEventSynchronize(a->ring_ev[b]));
+        ps::host_convert_f32(src + c0, a->ring[b], prec[m], len, threads, true);
+        PS_CUDA(cudaMemcpyAsync(slot + c0 * es, a->ring[b], len * es, cudaMemcpyHostToDevice, st));
+        PS_CUDA(cudaEventRecord(a->ring_ev[b], st));
+      }
+      a->pre[m] = 1;
+    } else {                                  // (a) single loop / (b) multithreaded SIMD
+      const bool simd = meth == PS_XFER_HOST_SIMD;
+      ps::host_convert_f32(src, a->pinned, prec[m], n, simd ? threads : 1, simd);
+      PS_CUDA(cudaMemcpyAsync(slot, a->pinned, n * es, cudaMemcpyHostToDevice, st));
+      PS_CUDA(cudaStreamSynchronize(st));     // the staging buffer is reused by the next object
+      a->pre[m] = 1;
+    }
+  }
+  PS_CUDA(cudaStreamSynchronize(st));
+  const double t_in = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  // ---- a2..a5 on the device
+  QPart *res = (QPart *)(a->ws + a->qres_off);
+  s = enqueue_config(a, prec, st, res, a->ev.data(), true);
+  for (int m = 0; m < M; m++) a->pre[m] = 0;
+  if (s != PS_OK) return s;
+  PS_CUDA(cudaStreamSynchronize(st));
+  // ---- outputs: D2H of the delivered (back-converted) outputs
+  const auto t1 = std::chrono::steady_clock::now();
+  if (host_outputs)
+    for (int m = 0; m < M; m++)
+      if (a->def->o[m].is_output && host_outputs[m])
+        PS_CUDA(cudaMemcpyAsync(host_outputs[m], a->orig_out[m], nelem(a, m) * 4, cudaMemcpyDeviceToHost, st));
+  PS_CUDA(cudaMemcpyAsync(a->host_res, res, sizeof(QPart), cudaMemcpyDeviceToHost, st));
+  PS_CUDA(cudaStreamSynchronize(st));
+  const double t_out = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t1).count();
+  uint64_t id = 0;
+  ps_config_encode(a, prec, &id);
+  fill_result(a, id, a->host_res[0], a->ev.data(), toq, out);
+  out->transfer_ms = (float)(t_in + t_out);
+  out->total_ms += out->transfer_ms;
   return PS_OK;
 }
 

@@ -6,6 +6,8 @@ namespace ps {
 
 // ------------------------------------------------------------ conversion (a2)
 ps_status convert_async(const void *src, int st, void *dst, int dt, size_t n, cudaStream_t stream);
+// host-side f32 -> dt conversion (host_convert.cpp; Fig. 3a/3b)
+void host_convert_f32(const float *src, void *dst, int dt, size_t n, int threads, bool simd);
 
 // ------------------------------------------------------- quality (a4 + a5)
 constexpr int QTHREADS = 256;
