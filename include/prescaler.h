@@ -187,6 +187,12 @@ typedef enum {
 /* simd != 0 uses F16C/AVX2 when the CPU has them.  Host pointers.            */
 PS_API ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, int threads,
                                  int simd);
+/* One object's {type conversion then transfer} with a method (the System     */
+/* Inspector's probe): host f32 array -> dev_dst in dst_type.  Methods */
+/* c and d need dev_stage (n*4 / n*2 bytes) for the device-side part.         */
+/* Synchronous; *ms = wall-clock milliseconds of conversion + transfer.       */
+PS_API ps_status ps_transfer(const float *host_src, void *dev_dst, int dst_type, size_t n,
+                             int method, int threads, void *dev_stage, void *stream, float *ms);
 /* Evaluate one configuration from HOST f32 inputs (host_inputs[m] for role   */
 /* in/inout, pinned memory recommended): per-object method `methods[m]`      */
 /* (NULL = all PS_XFER_DEVICE), `threads` host workers; the delivered f32     */

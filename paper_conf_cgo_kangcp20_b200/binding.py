@@ -29,6 +29,7 @@ SYMBOLS = [
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
     "ps_run_config", "ps_sweep", "ps_search", "ps_host_convert", "ps_run_config_host",
+    "ps_transfer",
 ]
 # type-conversion methods for host inputs (Fig. 3)
 XFER_DEVICE, XFER_HOST_LOOP, XFER_HOST_SIMD, XFER_PIPELINE, XFER_TRANSIENT = 0, 1, 2, 3, 4
@@ -117,6 +118,8 @@ def lib():
                                              ctypes.POINTER(PsSearchResult)]),
                 "ps_host_convert": (ctypes.c_int, [vp, vp, ctypes.c_int, ctypes.c_size_t, ctypes.c_int,
                                                    ctypes.c_int]),
+                "ps_transfer": (ctypes.c_int, [vp, vp, ctypes.c_int, ctypes.c_size_t, ctypes.c_int,
+                                               ctypes.c_int, vp, vp, ctypes.POINTER(ctypes.c_float)]),
                 "ps_run_config_host": (ctypes.c_int, [vp, ctypes.POINTER(ctypes.c_int),
                                                       ctypes.POINTER(ctypes.c_int), ctypes.POINTER(vp),
                                                       ctypes.POINTER(vp), ctypes.c_int, ctypes.c_double,
@@ -189,6 +192,15 @@ def ps_host_convert(src: np.ndarray, dst_type: int, threads: int = 0, simd: bool
     _check(lib().ps_host_convert(src.ctypes.data, out.ctypes.data, dst_type, src.size, threads,
                                  1 if simd else 0), "ps_host_convert")
     return out
+
+
+def ps_transfer(host_src, dev_dst, dst_type: int, n: int, method: int, threads: int = 0,
+                dev_stage=None, stream=None) -> float:
+    """One object's {conversion then transfer} with a Fig. 3 method; returns ms."""
+    ms = ctypes.c_float(0.0)
+    _check(lib().ps_transfer(_ptr(host_src), _ptr(dev_dst), dst_type, n, method, threads,
+                             _ptr(dev_stage), _stream(stream), ctypes.byref(ms)), "ps_transfer")
+    return float(ms.value)
 
 
 # -------------------------------------------------------------- (2) quality

@@ -100,6 +100,73 @@ using namespace ps;
 static constexpr int MAX_BATCH = 4096;
 static constexpr int NEV = 5;
 
+// Pinned host staging of the host-side conversion methods (Fig. 3a/b/d/e).
+struct XferScratch {
+  static constexpr size_t CH = (size_t)4 << 20;   // pipeline chunk: 4 Mi elements
+  void *pinned = nullptr;
+  size_t bytes = 0;
+  void *ring[2] = {nullptr, nullptr};
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  ps_status reserve(size_t need) {
+    if (need > bytes) {
+      if (pinned) cudaFreeHost(pinned);
+      pinned = nullptr;
+      bytes = 0;
+      PS_CUDA(cudaMallocHost(&pinned, need));
+      bytes = need;
+    }
+    if (!ring[0])
+      for (int k = 0; k < 2; k++) {
+        PS_CUDA(cudaMallocHost(&ring[k], CH * 8));
+        PS_CUDA(cudaEventCreateWithFlags(&ev[k], cudaEventDisableTiming));
+      }
+    return PS_OK;
+  }
+  ~XferScratch() {
+    if (pinned) cudaFreeHost(pinned);
+    for (int k = 0; k < 2; k++) {
+      if (ring[k]) cudaFreeHost(ring[k]);
+      if (ev[k]) cudaEventDestroy(ev[k]);
+    }
+  }
+};
+
+// Moves one f32 host array of n elements to the device in precision dt with a
+// Fig. 3 method.  Host methods (a, b, e) write dst directly; the device method
+// (c) writes f32 into stage and the transient method (d) writes fp16 into
+// stage -- the device-side conversion of those two is done by the caller (a2).
+// Synchronous with respect to the host staging buffers.
+static ps_status xfer_object(XferScratch &xs, const float *src, size_t n, int dt, int method,
+                             int threads, void *dst, void *stage, cudaStream_t st) {
+  const size_t es = dtype_size(dt);
+  if (method == PS_XFER_DEVICE) {
+    PS_CUDA(cudaMemcpyAsync(stage, src, n * 4, cudaMemcpyHostToDevice, st));
+    return PS_OK;
+  }
+  ps_status s = xs.reserve(method == PS_XFER_TRANSIENT ? n * 2 : (method == PS_XFER_PIPELINE ? 0 : n * es));
+  if (s != PS_OK) return s;
+  if (method == PS_XFER_TRANSIENT) {             // (d) host -> fp16 intermediate
+    ps::host_convert_f32(src, xs.pinned, PS_F16, n, threads, true);
+    PS_CUDA(cudaMemcpyAsync(stage, xs.pinned, n * 2, cudaMemcpyHostToDevice, st));
+    PS_CUDA(cudaStreamSynchronize(st));
+  } else if (method == PS_XFER_PIPELINE) {       // (e) chunked conversion overlapped with H2D
+    for (size_t c0 = 0, k = 0; c0 < n; c0 += XferScratch::CH, k++) {
+      const int b = (int)(k & 1);
+      const size_t len = std::min(XferScratch::CH, n - c0);
+      PS_CUDA(cudaEventSynchronize(xs.ev[b]));  // the slot's previous copy has left the buffer
+      ps::host_convert_f32(src + c0, xs.ring[b], dt, len, threads, true);
+      PS_CUDA(cudaMemcpyAsync((char *)dst + c0 * es, xs.ring[b], len * es, cudaMemcpyHostToDevice, st));
+      PS_CUDA(cudaEventRecord(xs.ev[b], st));
+    }
+  } else {                                       // (a) single loop / (b) multithreaded SIMD
+    const bool simd = method == PS_XFER_HOST_SIMD;
+    ps::host_convert_f32(src, xs.pinned, dt, n, simd ? threads : 1, simd);
+    PS_CUDA(cudaMemcpyAsync(dst, xs.pinned, n * es, cudaMemcpyHostToDevice, st));
+    PS_CUDA(cudaStreamSynchronize(st));          // the staging buffer is reused next
+  }
+  return PS_OK;
+}
+
 struct ps_app {
   const AppDef *def = nullptr;
   int kind = 0;
@@ -122,10 +189,7 @@ struct ps_app {
   // its data from: 0 = orig_in (device conversion), 1 = already in the slot at
   // c(m) (host conversion + H2D), 2 = fp16 intermediate in the transient region
   int pre[8] = {0};
-  void *pinned = nullptr;          // host staging (largest converted input)
-  size_t pinned_bytes = 0;
-  void *ring[2] = {nullptr, nullptr};
-  cudaEvent_t ring_ev[2] = {nullptr, nullptr};
+  XferScratch xs;                  // pinned host staging for the host methods
   // timing
   std::vector<cudaEvent_t> ev;
   QPart *host_res = nullptr;   // pinned, MAX_BATCH
@@ -133,11 +197,6 @@ struct ps_app {
   ~ps_app() {
     for (auto e : ev) cudaEventDestroy(e);
     if (host_res) cudaFreeHost(host_res);
-    if (pinned) cudaFreeHost(pinned);
-    for (int k = 0; k < 2; k++) {
-      if (ring[k]) cudaFreeHost(ring[k]);
-      if (ring_ev[k]) cudaEventDestroy(ring_ev[k]);
-    }
   }
 };
 
@@ -644,6 +703,34 @@ ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, i
   return PS_OK;
 }
 
+// One object's conversion + transfer with a Fig. 3 method (System Inspector probe).
+static thread_local XferScratch g_xs;
+ps_status ps_transfer(const float *host_src, void *dev_dst, int dst_type, size_t n, int method,
+                      int threads, void *dev_stage, void *stream, float *ms) {
+  if (!dtype_ok(dst_type) || method < PS_XFER_DEVICE || method > PS_XFER_TRANSIENT) {
+    set_error("ps_transfer: bad dtype or method");
+    return PS_ERR_INVALID;
+  }
+  if (n && (!host_src || !dev_dst)) { set_error("ps_transfer: null pointer"); return PS_ERR_INVALID; }
+  const bool staged = method == PS_XFER_DEVICE || method == PS_XFER_TRANSIENT;
+  if (n && staged && !dev_stage) { set_error("ps_transfer: this method needs dev_stage"); return PS_ERR_INVALID; }
+  if (threads <= 0) threads = (int)std::max(1u, std::thread::hardware_concurrency());
+  cudaStream_t st = (cudaStream_t)stream;
+  PS_CUDA(cudaStreamSynchronize(st));
+  const auto t0 = std::chrono::steady_clock::now();
+  if (n) {
+    ps_status s = xfer_object(g_xs, host_src, n, dst_type, method, threads, dev_dst, dev_stage, st);
+    if (s != PS_OK) return s;
+    if (staged) {   // the device-side part: f32 (c) or fp16 (d) -> dst_type
+      s = convert_async(dev_stage, method == PS_XFER_DEVICE ? PS_F32 : PS_F16, dev_dst, dst_type, n, st);
+      if (s != PS_OK) return s;
+    }
+  }
+  PS_CUDA(cudaStreamSynchronize(st));
+  if (ms) *ms = (float)std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return PS_OK;
+}
+
 // Whole-program evaluation from host inputs with per-object conversion methods
 // (Fig. 3 a-e); see prescaler.h.
 ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
@@ -657,9 +744,6 @@ ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
   if (threads <= 0) threads = (int)std::max(1u, std::thread::hardware_concurrency());
   cudaStream_t st = (cudaStream_t)stream;
   const int M = a->def->nobj;
-  constexpr size_t CH = (size_t)4 << 20;   // pipeline chunk: 4 Mi elements (16 MiB of f32)
-  // staging buffers (pinned, library-owned, grown on demand)
-  size_t need = 0;
   for (int m = 0; m < M; m++) {
     const int role = a->def->o[m].role;
     if (role != 0 && role != 2) continue;
@@ -668,21 +752,6 @@ ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
       set_error("ps_run_config_host: bad method or missing host input %d", m);
       return PS_ERR_INVALID;
     }
-    if (meth == PS_XFER_HOST_LOOP || meth == PS_XFER_HOST_SIMD) need = std::max(need, nelem(a, m) * dtype_size(prec[m]));
-    if (meth == PS_XFER_TRANSIENT) need = std::max(need, nelem(a, m) * 2);
-  }
-  if (need > a->pinned_bytes) {
-    if (a->pinned) cudaFreeHost(a->pinned);
-    a->pinned = nullptr;
-    a->pinned_bytes = 0;
-    PS_CUDA(cudaMallocHost(&a->pinned, need));
-    a->pinned_bytes = need;
-  }
-  if (!a->ring[0]) {
-    for (int k = 0; k < 2; k++) {
-      PS_CUDA(cudaMallocHost(&a->ring[k], CH * 8));
-      PS_CUDA(cudaEventCreateWithFlags(&a->ring_ev[k], cudaEventDisableTiming));
-    }
   }
   // ---- inputs: host conversion + H2D per object, in object order (wall clock)
   const auto t0 = std::chrono::steady_clock::now();
@@ -690,36 +759,14 @@ ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
     const int role = a->def->o[m].role;
     a->pre[m] = 0;
     if (role != 0 && role != 2) continue;
-    const int meth = methods ? methods[m] : PS_XFER_DEVICE;
-    const size_t n = nelem(a, m), es = dtype_size(prec[m]);
-    const float *src = (const float *)host_inputs[m];
-    char *slot = a->ws + a->slot_off[m];
-    if (meth == PS_XFER_DEVICE || (prec[m] == PS_F32 && role == 0 && meth != PS_XFER_TRANSIENT)) {
-      // (c): H2D at orig, the device converts in a2 (f32 inputs are used in place)
-      PS_CUDA(cudaMemcpyAsync((void *)a->orig_in[m], src, n * 4, cudaMemcpyHostToDevice, st));
-    } else if (meth == PS_XFER_TRANSIENT) {   // (d): host -> fp16, H2D fp16, device fp16 -> c(m)
-      ps::host_convert_f32(src, a->pinned, PS_F16, n, threads, true);
-      PS_CUDA(cudaMemcpyAsync(a->ws + a->trans_off[m], a->pinned, n * 2, cudaMemcpyHostToDevice, st));
-      PS_CUDA(cudaStreamSynchronize(st));
-      a->pre[m] = 2;
-    } else if (meth == PS_XFER_PIPELINE) {    // (e): chunked conversion overlapped with H2D
-      for (size_t c0 = 0, k = 0; c0 < n; c0 += CH, k++) {
-        const int b = (int)(k & 1);
-        const size_t len = std::min(CH, n - c0);
-        // the slot's previous copy (this or an earlier object) must have left the buffer
-        PS_CUDA(cudaEventSynchronize(a->ring_ev[b]));
-        ps::host_convert_f32(src + c0, a->ring[b], prec[m], len, threads, true);
-        PS_CUDA(cudaMemcpyAsync(slot + c0 * es, a->ring[b], len * es, cudaMemcpyHostToDevice, st));
-        PS_CUDA(cudaEventRecord(a->ring_ev[b], st));
-      }
-      a->pre[m] = 1;
-    } else {                                  // (a) single loop / (b) multithreaded SIMD
-      const bool simd = meth == PS_XFER_HOST_SIMD;
-      ps::host_convert_f32(src, a->pinned, prec[m], n, simd ? threads : 1, simd);
-      PS_CUDA(cudaMemcpyAsync(slot, a->pinned, n * es, cudaMemcpyHostToDevice, st));
-      PS_CUDA(cudaStreamSynchronize(st));     // the staging buffer is reused by the next object
-      a->pre[m] = 1;
-    }
+    int meth = methods ? methods[m] : PS_XFER_DEVICE;
+    // an f32 input already has its precision: H2D at orig, used in place by a2
+    if (prec[m] == PS_F32 && role == 0 && meth != PS_XFER_TRANSIENT) meth = PS_XFER_DEVICE;
+    void *stage = meth == PS_XFER_TRANSIENT ? (void *)(a->ws + a->trans_off[m]) : (void *)a->orig_in[m];
+    s = xfer_object(a->xs, (const float *)host_inputs[m], nelem(a, m), prec[m], meth, threads,
+                    a->ws + a->slot_off[m], stage, st);
+    if (s != PS_OK) return s;
+    a->pre[m] = meth == PS_XFER_DEVICE ? 0 : (meth == PS_XFER_TRANSIENT ? 2 : 1);
   }
   PS_CUDA(cudaStreamSynchronize(st));
   const double t_in = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();

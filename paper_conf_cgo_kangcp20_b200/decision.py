@@ -1,0 +1,198 @@
+"""PreScaler's Decision Maker on top of the C ABI (paper Sec. 4.2-4.4).
+
+* ``inspect`` -- the System Inspector's dynamic pass: the
+  throughput of {type conversion then transfer} for every method (Fig. 3 a-e,
+  ``ps_transfer``) x destination precision x array size, persisted as a JSON
+  "system information matrix".
+* ``best_method`` -- Alg. 2: for a transfer event, the method /
+  intermediate type with the least expected time among the candidates, from the
+  database only (no execution).
+* ``decide`` -- Alg. 1 per memory object, objects in descending order
+  of the time of their related events, starting from the pre-full-
+  precision configuration (Sec. 4.4.1): normal search in descending
+  precision with the best direct method (lines 2-13, stop at the first TOQ
+  failure), then the wildcard test with a transient intermediate type (lines
+  14-32: expected time = expected transfer time + the measured kernel time of the
+  target type; executed only if the failed type is the intermediate).
+  ``RunApp`` (line 8) is ``ps_run_config_host``.
+
+The native ``ps_search`` is the device-only variant (no transfer events).
+"""
+from __future__ import annotations
+
+import bisect
+import json
+import os
+import platform
+import statistics
+
+from . import binding as B
+
+METHODS = (B.XFER_DEVICE, B.XFER_HOST_LOOP, B.XFER_HOST_SIMD, B.XFER_PIPELINE, B.XFER_TRANSIENT)
+DIRECT = (B.XFER_DEVICE, B.XFER_HOST_LOOP, B.XFER_HOST_SIMD, B.XFER_PIPELINE)
+NAMES = {B.XFER_DEVICE: "device", B.XFER_HOST_LOOP: "host_loop", B.XFER_HOST_SIMD: "host_simd",
+         B.XFER_PIPELINE: "pipeline", B.XFER_TRANSIENT: "transient_f16"}
+SIZE = {B.F64: 8, B.F32: 4, B.F16: 2}
+
+
+# ------------------------------------------------------------------ inspector
+def inspect(sizes=(1 << 20, 1 << 23, 1 << 26), threads: int = 0, reps: int = 3, device=None,
+            methods=METHODS, path: str = None) -> dict:
+    """Measure ms of ps_transfer for every (method, dst precision, n)."""
+    import torch
+    dev = device or torch.device("cuda", torch.cuda.current_device())
+    nmax = max(sizes)
+    host = torch.rand(nmax, dtype=torch.float32).pin_memory()
+    dst = torch.empty(nmax * 8, dtype=torch.uint8, device=dev)
+    stage = torch.empty(nmax * 4, dtype=torch.uint8, device=dev)
+    entries = []
+    for n in sizes:
+        for dt in (B.F64, B.F32, B.F16):
+            for meth in methods:
+                B.ps_transfer(host, dst, dt, n, meth, threads, stage)      # warm-up
+                ms = statistics.median(B.ps_transfer(host, dst, dt, n, meth, threads, stage)
+                                       for _ in range(reps))
+                entries.append({"method": meth, "name": NAMES[meth], "dst": dt, "n": int(n),
+                                "ms": ms})
+    db = {"static": {"cpu": platform.processor() or platform.machine(), "cpu_cores": os.cpu_count(),
+                     "gpu": torch.cuda.get_device_name(dev), "threads": threads},
+          "entries": entries}
+    if path:
+        with open(path, "w") as f:
+            json.dump(db, f, indent=1)
+    return db
+
+
+def expected_ms(db: dict, method: int, dst: int, n: int) -> float:
+    """getExpectedTransferTime for one event: piecewise-linear in n over the
+    measured sizes, proportional beyond the largest (Alg. 1 line 20)."""
+    pts = sorted((e["n"], e["ms"]) for e in db["entries"] if e["method"] == method and e["dst"] == dst)
+    if not pts:
+        return float("inf")
+    ns = [p[0] for p in pts]
+    if n <= ns[0]:
+        return pts[0][1] * n / ns[0] if n < ns[0] else pts[0][1]
+    if n >= ns[-1]:
+        return pts[-1][1] * n / ns[-1]
+    k = bisect.bisect_left(ns, n)
+    (n0, t0), (n1, t1) = pts[k - 1], pts[k]
+    return t0 + (t1 - t0) * (n - n0) / (n1 - n0)
+
+
+def best_method(db: dict, n: int, target: int, intermediates=(B.F32,)):
+    """Alg. 2: (method, intermediate, expected ms) with the least expected time.
+    A candidate intermediate equal to the original (f32) or the target means a
+    direct conversion (any direct method); a lower-precision intermediate (f16)
+    for an f32/f64 target means the transient method."""
+    best = None
+    for inter in intermediates:
+        if inter in (B.F32, target):
+            cands = [(m, target) for m in DIRECT]
+        elif inter == B.F16 and target in (B.F32, B.F64):
+            cands = [(B.XFER_TRANSIENT, B.F16)]
+        else:
+            continue
+        for m, i in cands:
+            t = expected_ms(db, m, target, n)
+            if best is None or t < best[2]:
+                best = (m, i, t)
+    return best
+
+
+# ------------------------------------------------------------ decision maker
+def decide(app, host_inputs, db: dict, toq: float = 0.9, threads: int = 0, verify: bool = True):
+    """Alg. 1 over all objects with PFP initialisation.  Returns a dict with the chosen
+    precisions and methods, the final measured run, and the trial log."""
+    objs = app.objects
+    M = app.num_objects
+    inputs = [k for k, o in enumerate(objs) if o["role"] in (0, 2)]
+    log = []
+    cache = {}
+
+    def methods_for(prec, override=None):
+        meth = [B.XFER_DEVICE] * M
+        for k in inputs:
+            meth[k] = best_method(db, objs[k]["n"], prec[k])[0]
+        if override:
+            meth[override[0]] = override[1]
+        return meth
+
+    def run_app(prec, meth):                      # Alg. 1 line 8
+        key = (tuple(prec), tuple(meth))
+        if key not in cache:
+            r = app.run_config_host(prec, host_inputs, meth, threads=threads, toq=toq)
+            r["kernel_side_ms"] = r["total_ms"] - r["transfer_ms"]
+            cache[key] = r
+            log.append({"prec": list(prec), "methods": list(meth), "total_ms": r["total_ms"],
+                        "transfer_ms": r["transfer_ms"], "quality": r["quality"], "pass": r["pass"]})
+        return cache[key]
+
+    # Sec. 4.4.1 pre-full-precision scaling
+    cur, cur_m, cur_r = None, None, None
+    for t in (B.F64, B.F32, B.F16):
+        prec = [t] * M
+        meth = methods_for(prec)
+        r = run_app(prec, meth)
+        if r["pass"] and (cur_r is None or r["total_ms"] < cur_r["total_ms"]):
+            cur, cur_m, cur_r = prec, meth, r
+    if cur is None:
+        cur = [B.F64] * M
+        cur_m = methods_for(cur)
+        cur_r = run_app(cur, cur_m)
+    pfp = {"prec": list(cur), "methods": list(cur_m), "total_ms": cur_r["total_ms"]}
+
+    # objects in descending order of the time of their related events:
+    # expected transfer time for inputs, data volume at HBM speed otherwise
+    def weight(k):
+        n = objs[k]["n"]
+        if k in inputs:
+            return best_method(db, n, cur[k])[2]
+        return n * SIZE[cur[k]] / 6.5e9 * 1e3
+    order = sorted(range(M), key=lambda k: (-weight(k), k))
+
+    for k in order:
+        best, best_m, best_r = list(cur), list(cur_m), cur_r
+        accepted, failed, kernel_ms = [], None, {cur[k]: cur_r["kernel_side_ms"]}
+        for t in (B.F64, B.F32, B.F16):           # lines 2-13, descending precision
+            if t == cur[k]:
+                accepted.append(t)
+                continue
+            prec = list(cur)
+            prec[k] = t
+            meth = methods_for(prec)
+            r = run_app(prec, meth)
+            kernel_ms[t] = r["kernel_side_ms"]
+            if not r["pass"]:
+                failed = t
+                break
+            accepted.append(t)
+            if r["total_ms"] < best_r["total_ms"]:
+                best, best_m, best_r = prec, meth, r
+        # lines 14-32: wildcard test (transient intermediate) for input objects
+        if k in inputs:
+            wbest = None
+            for t in accepted:
+                inters = tuple(accepted) + ((failed,) if failed is not None else ())
+                m, inter, exp_t = best_method(db, objs[k]["n"], t, inters)
+                if m != B.XFER_TRANSIENT:
+                    continue
+                prec = list(cur)
+                prec[k] = t
+                meth = methods_for(prec, (k, m))
+                others = sum(best_method(db, objs[j]["n"], prec[j])[2] for j in inputs if j != k)
+                expected = exp_t + others + kernel_ms.get(t, float("inf"))   # line 20
+                if wbest is None or expected < wbest[2]:
+                    wbest = (prec, meth, expected, inter)
+            if wbest is not None and wbest[2] < best_r["total_ms"]:        # line 23
+                prec, meth, _, inter = wbest
+                ok = True
+                if verify or inter == failed:                                # lines 24-28
+                    ok = run_app(prec, meth)["pass"]
+                if ok:
+                    best, best_m = prec, meth
+                    best_r = run_app(prec, meth)
+        cur, cur_m, cur_r = best, best_m, best_r
+
+    return {"prec": list(cur), "methods": list(cur_m), "method_names": [NAMES[m] for m in cur_m],
+            "result": cur_r, "pfp": pfp, "trials": len(log), "log": log,
+            "space": 3 ** M}
