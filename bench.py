@@ -263,6 +263,38 @@ def cpu_baseline(args):
                           expo, factor)}
 
 
+# ------------------------------------------------------- whole program
+def whole_program(torch, B, apps, args):
+    """The paper's end metric: the Decision Maker's configuration (precisions +
+    conversion methods chosen from a System Inspector DB measured here) vs the original
+    program (every object f32, transferred as f32), both run from pinned host inputs
+    with ps_run_config_host (transfers included).  Not part of the timed value."""
+    from paper_conf_cgo_kangcp20_b200 import decision as D
+    t0 = time.time()
+    db = D.inspect(sizes=(1 << 20, 1 << 24, 1 << 26), reps=2)
+    out = {"inspector_s": None, "apps": {}}
+    out["inspector_s"] = round(time.time() - t0, 2)
+    out["best_methods_n2^26"] = {
+        {0: "f64", 1: "f32", 2: "f16"}[dt]: D.NAMES[D.best_method(db, 1 << 26, dt)[0]] for dt in (0, 1, 2)}
+    for a in apps:
+        app = a["app"]
+        host = [torch.from_numpy(x.reshape(-1)).pin_memory() if x is not None else None for x in a["ins"]]
+        m = app.num_objects
+        res = D.decide(app, host, db, toq=args.toq)
+        orig = [app.run_config_host([1] * m, host, [0] * m, toq=args.toq)["total_ms"] for _ in range(3)]
+        mine = [app.run_config_host(res["prec"], host, res["methods"], toq=args.toq)["total_ms"]
+                for _ in range(3)]
+        out["apps"][a["kind"]] = {
+            "original_f32_ms": round(float(np.median(orig)), 3),
+            "chosen": {"prec": res["prec"], "methods": res["method_names"]},
+            "chosen_ms": round(float(np.median(mine)), 3),
+            "speedup": round(float(np.median(orig) / np.median(mine)), 3),
+            "trials": res["trials"], "space": res["space"],
+            "quality": round(res["result"]["quality"], 6)}
+        del host
+    return out
+
+
 # ------------------------------------------------------------ conversion
 def conversion_sweep(torch, B, flush, reps=10):
     out = {}
@@ -302,6 +334,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-conversion", action="store_true")
+    ap.add_argument("--no-whole-program", action="store_true")
     ap.add_argument("--profile", action="store_true",
                     help="one untimed-warmup-free step for ncu launch lists (not a bench number)")
     args = ap.parse_args()
@@ -509,6 +542,10 @@ def main():
     else:
         roof, conv_roof = roof_a3, roof_a2
 
+    whole = None
+    if not args.no_whole_program and world == 1:
+        whole = whole_program(torch, B, apps, args)
+
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_baseline(args)
@@ -539,6 +576,7 @@ def main():
         "roofline_secondary": conv_roof,
         "conversion_gbs": conv,
         "speedup_vs_fp32_at_toq": speedup,
+        "whole_program": whole,
     }
     print(json.dumps(line), flush=True)
     if world > 1:
