@@ -344,6 +344,9 @@ static const app_def_t APPS[] = {
   {"gesummv", 5, 1, {"A", "B", "x", "y", "tmp"}, {0, 0, 0, 1, 3}, {0, 0, 0, 1, 0}},
   {"corr", 4, 2, {"data", "mean", "stddev", "symmat"}, {2, 3, 3, 1}, {0, 0, 0, 1}},
   {"covar", 3, 2, {"data", "mean", "symmat"}, {2, 3, 1}, {0, 0, 1}},
+  {"mvt", 5, 1, {"A", "x1", "x2", "y1", "y2"}, {0, 2, 2, 0, 0}, {0, 1, 1, 0, 0}},
+  {"syrk", 2, 2, {"A", "C"}, {0, 2}, {0, 1}},
+  {"conv2d", 2, 2, {"A", "B"}, {0, 1}, {0, 1}},
 };
 
 static const app_def_t *find_app(const char *kind) {
@@ -405,10 +408,19 @@ static void shapes(const app_def_t *a, const int64_t *d, int64_t rows[8], int64_
     rows[0] = d[0]; cols[0] = d[1];          /* data N x M */
     cols[1] = d[1]; cols[2] = d[1];          /* mean, stddev M */
     rows[3] = d[1]; cols[3] = d[1];          /* symmat M x M */
-  } else {                                   /* covar */
+  } else if (!strcmp(a->kind, "covar")) {    /* N rows, M cols */
     rows[0] = d[0]; cols[0] = d[1];
     cols[1] = d[1];
     rows[2] = d[1]; cols[2] = d[1];
+  } else if (!strcmp(a->kind, "mvt")) {      /* N */
+    rows[0] = d[0]; cols[0] = d[0];
+    cols[1] = d[0]; cols[2] = d[0]; cols[3] = d[0]; cols[4] = d[0];
+  } else if (!strcmp(a->kind, "syrk")) {     /* A: N x M, C: M x M */
+    rows[0] = d[0]; cols[0] = d[1];
+    rows[1] = d[1]; cols[1] = d[1];
+  } else {                                   /* conv2d: NI x NJ */
+    rows[0] = d[0]; cols[0] = d[1];
+    rows[1] = d[0]; cols[1] = d[1];
   }
 }
 
@@ -545,7 +557,61 @@ static void app_covar(obj_t *o, const int64_t *d) {
   syrk_upper(&o[0], &o[2], N, M, 0, (double)N - 1.0);             /* symmat */
 }
 
+/* MVT: x1 <- x1 + A y1 (row-dot, R5) ; x2 <- x2 + A^T y2 (column-sum, R5) */
+static void app_mvt(obj_t *o, const int64_t *d) {
+  size_t N = d[0], i;
+  int T1 = W3(o[0].type, o[1].type, o[3].type), T2 = W3(o[0].type, o[2].type, o[4].type);
+  for (i = 0; i < N; i++)
+    st(&o[1], i, t_add(T1, ld(&o[1], i), rowdot(T1, &o[0], i * N, N, &o[3])), T1);
+  for (i = 0; i < N; i++)
+    st(&o[2], i, t_add(T2, ld(&o[2], i), colsum(T2, &o[0], N, N, i, &o[4], 0)), T2);
+}
+
+/* SYRK (BLAS 'T' form, reading #23): C <- alpha A^T A + beta C over A: N x M,
+ * C_j1j2 = fma(alpha, sum_k A_kj1 A_kj2, beta C_j1j2) for j1 <= j2 (R3), mirrored */
+static void app_syrk(obj_t *o, const int64_t *d, const double *sc) {
+  size_t N = d[0], M = d[1], j1, j2;
+  int T = W2(o[0].type, o[1].type);
+  double al = t_lit(T, scalar_or(sc, 0, 32412.0)), be = t_lit(T, scalar_or(sc, 1, 2123.0));
+  for (j1 = 0; j1 < M; j1++)
+    for (j2 = j1; j2 < M; j2++) {
+      double acc = dot_chain(T, &o[0], j1, M, &o[0], j2, M, N);
+      double r = t_fma(T, al, acc, t_mul(T, be, ld(&o[1], j1 * M + j2)));
+      st(&o[1], j1 * M + j2, r, T);
+      st(&o[1], j2 * M + j1, r, T);
+    }
+}
+
+/* 2DCONV (reading #24): B_ij = c11 A(i-1,j-1) + c12 A(i,j-1) + c13 A(i+1,j-1)
+ *   + c21 A(i-1,j) + c22 A(i,j) + c23 A(i+1,j) + c31 A(i-1,j+1) + c32 A(i,j+1)
+ *   + c33 A(i+1,j+1), each product rounded in T, sums left to right (no
+ *   contraction, R4), for 1 <= i < NI-1, 1 <= j < NJ-1; border outputs +0. */
+static const double CONV2D_C[9] = {0.2, -0.3, 0.4, 0.5, 0.6, 0.7, -0.8, -0.9, 0.10};
+static double conv2d_at(int T, const obj_t *A, size_t NJ, size_t i, size_t j) {
+  static const int di[9] = {-1, 0, 1, -1, 0, 1, -1, 0, 1};
+  static const int dj[9] = {-1, -1, -1, 0, 0, 0, 1, 1, 1};
+  double acc = 0.0;
+  int k;
+  for (k = 0; k < 9; k++) {
+    double p = t_mul(T, t_lit(T, CONV2D_C[k]), ld(A, (i + di[k]) * NJ + (j + dj[k])));
+    acc = (k == 0) ? p : t_add(T, acc, p);
+  }
+  return acc;
+}
+static void app_conv2d(obj_t *o, const int64_t *d) {
+  size_t NI = d[0], NJ = d[1], i, j;
+  int T = W2(o[0].type, o[1].type);
+  for (i = 0; i < NI; i++)
+    for (j = 0; j < NJ; j++) {
+      int border = (i == 0 || j == 0 || i + 1 >= NI || j + 1 >= NJ);
+      st(&o[1], i * NJ + j, border ? 0.0 : conv2d_at(T, &o[0], NJ, i, j), T);
+    }
+}
+
 static int run_objects(const app_def_t *a, const int64_t *d, const double *sc, obj_t *o) {
+  if (!strcmp(a->kind, "mvt")) { app_mvt(o, d); return 0; }
+  if (!strcmp(a->kind, "syrk")) { app_syrk(o, d, sc); return 0; }
+  if (!strcmp(a->kind, "conv2d")) { app_conv2d(o, d); return 0; }
   if (!strcmp(a->kind, "gemm")) app_gemm(o, d, sc);
   else if (!strcmp(a->kind, "2mm")) app_2mm(o, d);
   else if (!strcmp(a->kind, "3mm")) app_3mm(o, d);
@@ -768,6 +834,34 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
       double tv = round_to(prec[4], rowdot(T1, &in[0], i * N, N, &in[2]), T1);
       double yv = round_to(prec[3], rowdot(T2, &in[1], i * N, N, &in[2]), T2);
       vals[k] = round_to(prec[3], t_fma(T3, al, tv, t_mul(T3, be, yv)), T3);
+    }
+  } else if (!strcmp(kind, "mvt")) {
+    size_t N = d[0];
+    int T1 = W3(prec[0], prec[1], prec[3]), T2 = W3(prec[0], prec[2], prec[4]);
+    for (k = 0; k < n; k++) {
+      size_t i = cols[k];
+      if (m == 1)
+        vals[k] = round_to(prec[1], t_add(T1, ld(&in[1], i), rowdot(T1, &in[0], i * N, N, &in[3])), T1);
+      else
+        vals[k] = round_to(prec[2], t_add(T2, ld(&in[2], i), colsum(T2, &in[0], N, N, i, &in[4], 0)), T2);
+    }
+  } else if (!strcmp(kind, "syrk")) {
+    size_t N = d[0], M = d[1];
+    int T = W2(prec[0], prec[1]);
+    double al = t_lit(T, scalar_or(sc, 0, 32412.0)), be = t_lit(T, scalar_or(sc, 1, 2123.0));
+    for (k = 0; k < n; k++) {
+      size_t j1 = rows[k], j2 = cols[k];
+      if (j1 > j2) { size_t s = j1; j1 = j2; j2 = s; }   /* mirrored lower triangle */
+      double acc = dot_chain(T, &in[0], j1, M, &in[0], j2, M, N);
+      vals[k] = round_to(prec[1], t_fma(T, al, acc, t_mul(T, be, ld(&in[1], j1 * M + j2))), T);
+    }
+  } else if (!strcmp(kind, "conv2d")) {
+    size_t NI = d[0], NJ = d[1];
+    int T = W2(prec[0], prec[1]);
+    for (k = 0; k < n; k++) {
+      size_t i = rows[k], j = cols[k];
+      int border = (i == 0 || j == 0 || i + 1 >= NI || j + 1 >= NJ);
+      vals[k] = round_to(prec[1], border ? 0.0 : conv2d_at(T, &in[0], NJ, i, j), T);
     }
   } else {                                  /* corr / covar: symmat entries */
     int corr = !strcmp(kind, "corr");

@@ -52,7 +52,9 @@ def test_object_tables(oracle_lib):
 
 # ----------------------------------------------------- f64 vs numpy textbook
 DIMS = {"gemm": [13, 17, 11], "2mm": [9, 14, 11, 7], "3mm": [6, 9, 8, 10, 7],
-        "atax": [37, 45], "bicg": [41, 33], "gesummv": [29], "corr": [40, 23], "covar": [35, 19]}
+        "atax": [37, 45], "bicg": [41, 33], "gesummv": [29], "corr": [40, 23], "covar": [35, 19],
+        "mvt": [43], "syrk": [31, 18], "conv2d": [17, 23]}
+CONV2D_C = [0.2, -0.3, 0.4, 0.5, 0.6, 0.7, -0.8, -0.9, 0.10]
 
 
 def numpy_ref(kind, ins, objs, scalars=None):
@@ -83,6 +85,22 @@ def numpy_ref(kind, ins, objs, scalars=None):
         return {3: c}
     if kind == "covar":
         return {2: np.cov(A[0], rowvar=False)}
+    if kind == "mvt":
+        return {1: (A[1][0] + A[0] @ A[3][0])[None, :], 2: (A[2][0] + A[0].T @ A[4][0])[None, :]}
+    if kind == "syrk":      # BLAS 'T' form; the result's lower triangle mirrors the upper
+        al, be = scalars or (32412.0, 2123.0)
+        cu = np.triu(A[1])
+        c = cu + np.triu(cu, 1).T
+        return {1: al * (A[0].T @ A[0]) + be * c}
+    if kind == "conv2d":
+        a = A[0]
+        b = np.zeros_like(a)
+        di = [-1, 0, 1] * 3
+        dj = [-1] * 3 + [0] * 3 + [1] * 3
+        ni, nj = a.shape
+        for c, x, y in zip(CONV2D_C, di, dj):
+            b[1:-1, 1:-1] += c * a[1 + x:ni - 1 + x, 1 + y:nj - 1 + y]
+        return {1: b}
     raise KeyError(kind)
 
 
@@ -137,7 +155,7 @@ def _fits(v, p):
     return np.all(np.abs(v) <= lim)
 
 
-@pytest.mark.parametrize("kind", ["gemm", "2mm", "3mm", "atax", "bicg", "gesummv"])
+@pytest.mark.parametrize("kind", ["gemm", "2mm", "3mm", "atax", "bicg", "gesummv", "mvt", "syrk"])
 def test_exact_integer_results_every_config(oracle_lib, kind):
     """With small non-negative integer inputs every partial sum is an integer
     bounded by the final value, so every configuration whose objects can hold
@@ -148,7 +166,9 @@ def test_exact_integer_results_every_config(oracle_lib, kind):
     dims = {"atax": [300, 77], "bicg": [270, 93], "gesummv": [75]}.get(kind, DIMS[kind])
     objs = oracle.app_objects(kind, dims)
     ins = _exact_ints(kind, dims, objs, rng)
-    sc = (2.0, 3.0) if kind in ("gemm", "gesummv") else None
+    sc = (2.0, 3.0) if kind in ("gemm", "gesummv", "syrk") else None
+    if kind == "syrk":        # C must be symmetric for the textbook form to apply
+        ins[1] = np.triu(ins[1]) + np.triu(ins[1], 1).T
     exact = {m: np.rint(v) for m, v in numpy_ref(kind, ins, objs, sc).items()}
     n_checked = 0
     for prec in itertools.product([F64, F32, F16], repeat=len(objs)):

@@ -9,7 +9,8 @@ import oracle
 from paper_conf_cgo_kangcp20_b200 import inputs as gen
 
 CASES = {"gemm": [37, 29, 41], "2mm": [19, 23, 17, 21], "3mm": [11, 13, 9, 15, 10],
-         "atax": [300, 77], "bicg": [270, 93], "gesummv": [75], "corr": [60, 17], "covar": [55, 13]}
+         "atax": [300, 77], "bicg": [270, 93], "gesummv": [75], "corr": [60, 17], "covar": [55, 13],
+         "mvt": [301], "syrk": [23, 14], "conv2d": [15, 21]}
 
 
 @pytest.mark.parametrize("kind", sorted(CASES))
