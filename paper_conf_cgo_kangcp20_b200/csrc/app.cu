@@ -79,10 +79,14 @@ static const AppDef kApps[] = {
     {"gesummv", 5, 1, {{"A", 0, 0}, {"B", 0, 0}, {"x", 0, 0}, {"y", 1, 1}, {"tmp", 3, 0}}},
     {"corr", 4, 2, {{"data", 2, 0}, {"mean", 3, 0}, {"stddev", 3, 0}, {"symmat", 1, 1}}},
     {"covar", 3, 2, {{"data", 2, 0}, {"mean", 3, 0}, {"symmat", 1, 1}}},
+    {"mvt", 5, 1, {{"A", 0, 0}, {"x1", 2, 1}, {"x2", 2, 1}, {"y1", 0, 0}, {"y2", 0, 0}}},
+    {"syrk", 2, 2, {{"A", 0, 0}, {"C", 2, 1}}},
+    {"conv2d", 2, 2, {{"A", 0, 0}, {"B", 1, 1}}},
 };
-enum AppKind { K_GEMM, K_2MM, K_3MM, K_ATAX, K_BICG, K_GESUMMV, K_CORR, K_COVAR };
+enum AppKind { K_GEMM, K_2MM, K_3MM, K_ATAX, K_BICG, K_GESUMMV, K_CORR, K_COVAR, K_MVT, K_SYRK,
+               K_CONV2D };
 // statements that read or write each object (for ps_search's object order)
-static const int kTouch[8][8] = {
+static const int kTouch[11][8] = {
     {1, 1, 1},                  // gemm: C <- aAB + bC
     {1, 1, 2, 1, 1},            // 2mm
     {1, 1, 1, 1, 2, 2, 1},      // 3mm
@@ -91,6 +95,9 @@ static const int kTouch[8][8] = {
     {1, 1, 2, 2, 2},            // gesummv
     {4, 3, 2, 1},               // corr
     {3, 2, 1},                  // covar
+    {2, 1, 1, 1, 1},            // mvt
+    {1, 1},                     // syrk
+    {1, 1},                     // conv2d
 };
 
 }  // namespace ps
@@ -227,6 +234,11 @@ void shapes(ps_app *a) {
       break;
     case K_CORR: set(0, d[0], d[1]); set(1, 1, d[1]); set(2, 1, d[1]); set(3, d[1], d[1]); break;
     case K_COVAR: set(0, d[0], d[1]); set(1, 1, d[1]); set(2, d[1], d[1]); break;
+    case K_MVT:
+      set(0, d[0], d[0]); set(1, 1, d[0]); set(2, 1, d[0]); set(3, 1, d[0]); set(4, 1, d[0]);
+      break;
+    case K_SYRK: set(0, d[0], d[1]); set(1, d[1], d[1]); break;
+    case K_CONV2D: set(0, d[0], d[1]); set(1, d[0], d[1]); break;
   }
 }
 
@@ -241,7 +253,7 @@ void layout(ps_app *a) {
   size_t pb = 0;
   if (a->kind == K_ATAX || a->kind == K_BICG || a->kind == K_CORR || a->kind == K_COVAR)
     pb = tile_partial_bytes(a->d[0], a->d[1]);
-  if (a->kind == K_GESUMMV) pb = tile_partial_bytes(a->d[0], a->d[0]);
+  if (a->kind == K_GESUMMV || a->kind == K_MVT) pb = tile_partial_bytes(a->d[0], a->d[0]);
   a->partial_off = off;
   off = align_up(off + pb, 256);
   int nout = 0;
@@ -291,6 +303,10 @@ ps_status syrk(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double 
   g.B = MatDesc{c.ptr[data], c.prec[data], M, 1};   // B(i, j2) = data[i][j2]
   g.C = c.ptr[sym]; g.c_type = c.prec[sym]; g.ldc = M;
   g.epi = epi; g.div = div;
+  if (epi == EPI_AXPBY) {   // SYRK app: C <- alpha data^T data + beta C (C read in place)
+    g.Cin = c.ptr[sym]; g.cin_type = c.prec[sym];
+    g.alpha = c.a->sc[0]; g.beta = c.a->sc[1];
+  }
   g.upper_only = 1;
   g.T = compute_type({c.prec[data], c.prec[sym]});
   ps_status s = contraction(c, g);
@@ -364,6 +380,15 @@ ps_status run_statements(Ctx &c) {
       S_(syrk(c, 0, 2, d[0], d[1], EPI_DIV, n - 1.0, 0));
       break;
     }
+    case K_MVT:   // x1 <- x1 + A y1 ; x2 <- x2 + A^T y2   (one pass over A)
+      S_(mvt_async(P[0], p[0], d[0], P[1], p[1], P[2], p[2], P[3], p[3], P[4], p[4], partial, c.st));
+      break;
+    case K_SYRK:  // C <- alpha A^T A + beta C (upper tiles, mirrored)
+      S_(syrk(c, 0, 1, d[0], d[1], EPI_AXPBY, 0.0, 0));
+      break;
+    case K_CONV2D:
+      S_(conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st));
+      break;
   }
 #undef S_
   return PS_OK;
@@ -511,8 +536,9 @@ ps_status ps_app_create(const char *kind, const int64_t *dims, int ndims, const 
   if (k == K_GEMM) { a->sc[0] = 32412.0; a->sc[1] = 2123.0; }
   if (k == K_GESUMMV) { a->sc[0] = 43532.0; a->sc[1] = 12313.0; }
   if (k == K_CORR) { a->sc[0] = 0.005; }
+  if (k == K_SYRK) { a->sc[0] = 32412.0; a->sc[1] = 2123.0; }
   if (scalars) {
-    if (k == K_GEMM || k == K_GESUMMV) { a->sc[0] = scalars[0]; a->sc[1] = scalars[1]; }
+    if (k == K_GEMM || k == K_GESUMMV || k == K_SYRK) { a->sc[0] = scalars[0]; a->sc[1] = scalars[1]; }
     if (k == K_CORR) a->sc[0] = scalars[0];
   }
   shapes(a);

@@ -68,7 +68,12 @@ ps_status bicg_async(const void *A, int ta, int64_t lda, const void *r, int tr, 
 //   mode 0: p = fma(A_ij, w_i, p)   mode 1: p = p + A_ij   mode 2: d = A_ij - w_j, p = fma(d, d, p)
 // finalize: 0 plain, 1 total / n, 2 stddev (sqrt(total / n), <= eps -> 1)
 enum ColMode { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
-enum ColFin { FIN_PLAIN = 0, FIN_MEAN = 1, FIN_STDDEV = 2 };
+enum ColFin { FIN_PLAIN = 0, FIN_MEAN = 1, FIN_STDDEV = 2, FIN_ADD = 3 /* out = out_old + total */ };
+// MVT in one pass over A: x1 <- x1 + A y1, x2 <- x2 + A^T y2 (n x n)
+ps_status mvt_async(const void *A, int ta, int64_t n, void *x1, int t1, void *x2, int t2,
+                    const void *y1, int ty1, const void *y2, int ty2, void *partial, cudaStream_t st);
+// 2DCONV 3x3 stencil (reading #24): B_ij = sum of 9 rounded products, left to right; border +0
+ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, cudaStream_t st);
 ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
                        int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
                        double eps, void *partial, cudaStream_t st);

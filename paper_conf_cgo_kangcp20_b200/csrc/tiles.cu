@@ -193,17 +193,19 @@ __global__ void __launch_bounds__(256) colsum_finalize_kernel(const T *__restric
     total = sqrt(total / n);
     if (total <= eps) total = T(1);
   }
+  if (FIN == FIN_ADD) total = Ld<SO, T>::get(out, (size_t)j) + total;   // MVT: x2 + A^T y2
   St<SO, T>::put(out, (size_t)j, total);
 }
 
 template <class T, class SO>
 __global__ void __launch_bounds__(256) rowdot_finalize_kernel(const T *__restrict__ qpart,
                                                               raw_t<SO> *__restrict__ out,
-                                                              int64_t rows, int64_t ntiles) {
+                                                              int64_t rows, int64_t ntiles, int add) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= rows) return;
   T total = qpart[i];
   for (int64_t t = 1; t < ntiles; t++) total = total + qpart[t * rows + i];   // tiles in order
+  if (add) total = Ld<SO, T>::get(out, (size_t)i) + total;                   // MVT: x1 + A y1
   St<SO, T>::put(out, (size_t)i, total);
 }
 
@@ -288,6 +290,9 @@ static ps_status colsum_finalize(const TileArgs &a, void *out, int tout, int fin
     if (fin == FIN_PLAIN)
       colsum_finalize_kernel<T, SO, FIN_PLAIN><<<fb, 256, 0, st>>>(sp, (raw_t<SO> *)out, a.cols,
                                                                   a.nchunks, (T)n, (T)eps);
+    else if (fin == FIN_ADD)
+      colsum_finalize_kernel<T, SO, FIN_ADD><<<fb, 256, 0, st>>>(sp, (raw_t<SO> *)out, a.cols,
+                                                                a.nchunks, (T)n, (T)eps);
     else if (fin == FIN_MEAN)
       colsum_finalize_kernel<T, SO, FIN_MEAN><<<fb, 256, 0, st>>>(sp, (raw_t<SO> *)out, a.cols,
                                                                  a.nchunks, (T)n, (T)eps);
@@ -300,12 +305,12 @@ static ps_status colsum_finalize(const TileArgs &a, void *out, int tout, int fin
 }
 
 template <class T>
-static ps_status rowdot_finalize(const TileArgs &a, void *out, int tout, cudaStream_t st) {
+static ps_status rowdot_finalize(const TileArgs &a, void *out, int tout, cudaStream_t st, int add = 0) {
   const unsigned fb = (unsigned)((a.rows + 255) / 256);
   return dispatch_store(tout, [&](auto so) -> ps_status {
     using SO = decltype(so);
     rowdot_finalize_kernel<T, SO><<<fb, 256, 0, st>>>((const T *)a.qpart, (raw_t<SO> *)out, a.rows,
-                                                      a.ntiles);
+                                                      a.ntiles, add);
     PS_CHECK_LAUNCH("rowdot_finalize_kernel");
     return PS_OK;
   });
@@ -342,6 +347,24 @@ ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw
   if (s != PS_OK) return s;
   return T == PS_F64 ? colsum_finalize<double>(a, out, tout, fin, n, eps, st)
                      : colsum_finalize<float>(a, out, tout, fin, n, eps, st);
+}
+
+// MVT in one pass over A: x1 <- x1 + A y1 (row dots), x2 <- x2 + A^T y2 (column sums)
+ps_status mvt_async(const void *A, int ta, int64_t n, void *x1, int t1, void *x2, int t2,
+                    const void *y1, int ty1, const void *y2, int ty2, void *partial, cudaStream_t st) {
+  if (n <= 0) return PS_OK;
+  TileArgs a = make_args(A, ta, n, n, n, partial);
+  a.w = y2;
+  a.tw = ty2;
+  a.x = y1;
+  a.tx = ty1;
+  const int TC = compute_type({ta, t2, ty2}), TR = compute_type({ta, t1, ty1});
+  ps_status e = tile_dispatch<COL_DOT, true>(a, ta, TC, TR, st);
+  if (e != PS_OK) return e;
+  e = TC == PS_F64 ? colsum_finalize<double>(a, x2, t2, FIN_ADD, 0, 0, st)
+                   : colsum_finalize<float>(a, x2, t2, FIN_ADD, 0, 0, st);
+  if (e != PS_OK) return e;
+  return TR == PS_F64 ? rowdot_finalize<double>(a, x1, t1, st, 1) : rowdot_finalize<float>(a, x1, t1, st, 1);
 }
 
 ps_status bicg_async(const void *A, int ta, int64_t lda, const void *r, int tr, void *s, int ts,

@@ -49,6 +49,12 @@ def _statements(kind, d):
                 ("mm", 0, 0, 3, (d[1], d[1], d[0] / 2.0))]
     if kind == "covar":
         return [("mv", 0, [0, 1]), ("ew", [0, 1]), ("mm", 0, 0, 2, (d[1], d[1], d[0] / 2.0))]
+    if kind == "mvt":
+        return [("mv", 0, [0, 1, 2, 3, 4])]
+    if kind == "syrk":
+        return [("mm", 0, 0, 1, (d[1], d[1], d[0] / 2.0))]
+    if kind == "conv2d":
+        return [("ew", [0, 1])]
     raise KeyError(kind)
 
 

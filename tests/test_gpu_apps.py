@@ -98,6 +98,12 @@ SIMT_CASES = [
     ("corr", [257, 33], "image", None),
     ("covar", [260, 90], "random", None),
     ("covar", [511, 37], "default", None),
+    ("mvt", [600], "random", None),
+    ("mvt", [2051], "default", None),
+    ("syrk", [260, 70], "random", (1.5, 1.2)),
+    ("syrk", [129, 257], "default", None),
+    ("conv2d", [200, 300], "random", None),
+    ("conv2d", [37, 65], "image", None),
 ]
 
 

@@ -95,6 +95,24 @@ def test_syrk_tc_bound(torch, kind, dims, prec):
     assert abs(r["quality"] - ro["quality"]) <= 1e-3
 
 
+@pytest.mark.parametrize("dims,c_prec", [([264, 136], B.F32), ([520, 264], B.F16)])
+def test_syrk_app_tc_bound(torch, dims, c_prec):
+    """SYRK app: C <- alpha A^T A + beta C on tcgen05 (A fp16, M-major operand)."""
+    sc = (1.5, 1.2)
+    app, ins, oref = setup(torch, "syrk", dims, "random", sc)
+    prec = [B.F16, c_prec]
+    r = app.run_config(prec)
+    ro, delivered = oracle.evaluate("syrk", dims, prec, ins, oref, sc)
+    M = dims[1]
+    got = app.outputs[1].cpu().numpy().astype(np.float64).reshape(M, M)
+    want = delivered[1].astype(np.float64).reshape(M, M)
+    a16 = np.abs(oracle.run_config("syrk", dims, prec, ins, sc)[0].astype(np.float64))
+    bound = sc[0] * 2 * gamma(dims[0]) * (a16.T @ a16) + 2 * ulp(want, np.float16 if c_prec == B.F16 else np.float32)
+    assert np.array_equal(got, got.T)
+    assert np.all(np.abs(got - want) <= bound)
+    assert abs(r["quality"] - ro["quality"]) <= 1e-3
+
+
 @pytest.mark.parametrize("kind,dims", [("2mm", [136, 264, 200, 72]), ("3mm", [136, 72, 200, 64, 128])])
 def test_chain_tc_relative(torch, kind, dims):
     """Every config of the chain apps with tensor cores enabled: fp16 statements
