@@ -43,6 +43,10 @@ WORKLOADS = {
     "contract": [("2mm", [8192])],
     "contract3mm": [("3mm", [8192])],
     "corr": [("corr", [8192, 8192]), ("covar", [8192, 8192])],
+    # SURVEY §8(f) NEXT #3 shapes at the mat-vec / contraction sizes of BASELINE
+    "mvt": [("mvt", [16384])],
+    "stencil": [("conv2d", [16384, 16384])],
+    "syrk": [("syrk", [8192, 8192])],
 }
 SIZE = {0: 8, 1: 4, 2: 2}
 # CPU-oracle samples: (reduced dimension, work exponent) -- the oracle needs ~40 s
@@ -50,7 +54,7 @@ SIZE = {0: 8, 1: 4, 2: 2}
 # the reduced size and extrapolate throughput by (N_sample / N)^exponent (O(N^2)
 # mat-vec, O(N^3) contractions); labelled "extrapolated" in the JSON.
 CPU_SAMPLE = {"matvec": (8192, 2), "gemm64": (None, 0), "contract": (384, 3), "contract3mm": (256, 3),
-              "corr": (512, 3)}
+              "corr": (512, 3), "mvt": (8192, 2), "stencil": (4096, 2), "syrk": (512, 3)}
 
 
 def log(*a):
@@ -124,6 +128,11 @@ def kernel_bytes(kind, dims, prec):
     if kind == "gesummv":
         return n * n * (SIZE[prec[0]] + SIZE[prec[1]]) + n * (SIZE[prec[2]] + 3 * SIZE[prec[3]] +
                                                             2 * SIZE[prec[4]])
+    if kind == "mvt":      # one pass over A; x1, x2 read and written, y1, y2 read
+        return n * n * SIZE[prec[0]] + n * (2 * SIZE[prec[1]] + 2 * SIZE[prec[2]] + SIZE[prec[3]] +
+                                            SIZE[prec[4]])
+    if kind == "conv2d":   # A read once, B written once
+        return dims[0] * dims[1] * (SIZE[prec[0]] + SIZE[prec[1]])
     return None
 
 
@@ -138,6 +147,8 @@ def _contractions(kind, d):
         return [(0, 1, 4, d[0], d[1], d[2]), (2, 3, 5, d[1], d[3], d[4]), (4, 5, 6, d[0], d[3], d[1])]
     if kind in ("corr", "covar"):
         return [(0, 0, 3 if kind == "corr" else 2, d[1], d[1], d[0] / 2.0)]
+    if kind == "syrk":
+        return [(0, 0, 1, d[1], d[1], d[0] / 2.0)]
     return []
 
 

@@ -81,8 +81,7 @@ __global__ void __launch_bounds__(QTHREADS) backconv_quality_kernel(
   double sum = 0.0, mx = 0.0;
   unsigned long long nf = 0;
   const size_t stride = (size_t)gridDim.x * QTHREADS;
-  for (size_t i = (size_t)blockIdx.x * QTHREADS + threadIdx.x; i < n; i += stride) {
-    const raw_t<S> v = out[i];
+  auto one = [&](size_t i, raw_t<S> v, double r) {
     double o;
     if (DELIVER) {
       const float d = Deliver<S>::f(v);
@@ -91,7 +90,42 @@ __global__ void __launch_bounds__(QTHREADS) backconv_quality_kernel(
     } else {
       o = Deliver<S>::exact(v);
     }
-    qual_elem(o, __ldg(ref + i), sum, mx, nf);
+    qual_elem(o, r, sum, mx, nf);
+  };
+  // 4 consecutive elements per thread per step: 16-byte loads of ref (2 x double2)
+  // and of out (f32) / 8-byte (f16) / 2 x 16-byte (f64) when everything is aligned
+  const bool vec = ((uintptr_t)out % 16 == 0) && ((uintptr_t)ref % 16 == 0) &&
+                   (!DELIVER || (uintptr_t)delivered % 16 == 0);
+  size_t i = ((size_t)blockIdx.x * QTHREADS + threadIdx.x) * 4;
+  if (vec) {
+    for (; i + 4 <= n; i += stride * 4) {
+      const double2 r0 = __ldg(reinterpret_cast<const double2 *>(ref + i));
+      const double2 r1 = __ldg(reinterpret_cast<const double2 *>(ref + i) + 1);
+      raw_t<S> v[4];
+#pragma unroll
+      for (int k = 0; k < 4; k++) v[k] = out[i + k];
+      if (DELIVER) {
+        float4 d;
+        d.x = Deliver<S>::f(v[0]);
+        d.y = Deliver<S>::f(v[1]);
+        d.z = Deliver<S>::f(v[2]);
+        d.w = Deliver<S>::f(v[3]);
+        *reinterpret_cast<float4 *>(delivered + i) = d;
+        qual_elem((double)d.x, r0.x, sum, mx, nf);
+        qual_elem((double)d.y, r0.y, sum, mx, nf);
+        qual_elem((double)d.z, r1.x, sum, mx, nf);
+        qual_elem((double)d.w, r1.y, sum, mx, nf);
+      } else {
+        qual_elem(Deliver<S>::exact(v[0]), r0.x, sum, mx, nf);
+        qual_elem(Deliver<S>::exact(v[1]), r0.y, sum, mx, nf);
+        qual_elem(Deliver<S>::exact(v[2]), r1.x, sum, mx, nf);
+        qual_elem(Deliver<S>::exact(v[3]), r1.y, sum, mx, nf);
+      }
+    }
+    for (; i < n; i++) one(i, out[i], __ldg(ref + i));   // ragged tail (this thread's last group)
+  } else {
+    for (size_t e = (size_t)blockIdx.x * QTHREADS + threadIdx.x; e < n; e += stride)
+      one(e, out[e], __ldg(ref + e));
   }
   block_reduce3(sum, mx, nf, s_sum, s_mx, s_nf);
   if (threadIdx.x == 0) parts[blockIdx.x] = QPart{sum, mx, nf};
