@@ -347,6 +347,9 @@ static const app_def_t APPS[] = {
   {"mvt", 5, 1, {"A", "x1", "x2", "y1", "y2"}, {0, 2, 2, 0, 0}, {0, 1, 1, 0, 0}},
   {"syrk", 2, 2, {"A", "C"}, {0, 2}, {0, 1}},
   {"conv2d", 2, 2, {"A", "B"}, {0, 1}, {0, 1}},
+  {"syr2k", 3, 2, {"A", "B", "C"}, {0, 0, 2}, {0, 0, 1}},
+  {"conv3d", 2, 3, {"A", "B"}, {0, 1}, {0, 1}},
+  {"fdtd2d", 4, 3, {"fict", "ex", "ey", "hz"}, {0, 2, 2, 2}, {0, 1, 1, 1}},
 };
 
 static const app_def_t *find_app(const char *kind) {
@@ -418,9 +421,21 @@ static void shapes(const app_def_t *a, const int64_t *d, int64_t rows[8], int64_
   } else if (!strcmp(a->kind, "syrk")) {     /* A: N x M, C: M x M */
     rows[0] = d[0]; cols[0] = d[1];
     rows[1] = d[1]; cols[1] = d[1];
-  } else {                                   /* conv2d: NI x NJ */
+  } else if (!strcmp(a->kind, "conv2d")) {   /* NI x NJ */
     rows[0] = d[0]; cols[0] = d[1];
     rows[1] = d[0]; cols[1] = d[1];
+  } else if (!strcmp(a->kind, "syr2k")) {    /* A, B: N x M; C: M x M */
+    rows[0] = d[0]; cols[0] = d[1];
+    rows[1] = d[0]; cols[1] = d[1];
+    rows[2] = d[1]; cols[2] = d[1];
+  } else if (!strcmp(a->kind, "conv3d")) {   /* NI x (NJ NK) */
+    rows[0] = d[0]; cols[0] = d[1] * d[2];
+    rows[1] = d[0]; cols[1] = d[1] * d[2];
+  } else {                                   /* fdtd2d: TMAX, NX, NY */
+    cols[0] = d[0];
+    rows[1] = d[1]; cols[1] = d[2];
+    rows[2] = d[1]; cols[2] = d[2];
+    rows[3] = d[1]; cols[3] = d[2];
   }
 }
 
@@ -608,7 +623,91 @@ static void app_conv2d(obj_t *o, const int64_t *d) {
     }
 }
 
+/* SYR2K (BLAS 'T' form, reading #25): C <- alpha A^T B + beta C ; C <- alpha B^T A + C
+ * (two statements, each an R3 chain and an RNE store of C) over A, B: N x M */
+static void app_syr2k(obj_t *o, const int64_t *d, const double *sc) {
+  size_t N = d[0], M = d[1], i, j;
+  int T = W3(o[0].type, o[1].type, o[2].type);
+  double al = t_lit(T, scalar_or(sc, 0, 32412.0)), be = t_lit(T, scalar_or(sc, 1, 2123.0));
+  for (i = 0; i < M; i++)
+    for (j = 0; j < M; j++) {
+      double s1 = dot_chain(T, &o[0], i, M, &o[1], j, M, N);
+      st(&o[2], i * M + j, t_fma(T, al, s1, t_mul(T, be, ld(&o[2], i * M + j))), T);
+    }
+  for (i = 0; i < M; i++)
+    for (j = 0; j < M; j++) {
+      double s2 = dot_chain(T, &o[1], i, M, &o[0], j, M, N);
+      st(&o[2], i * M + j, t_fma(T, al, s2, ld(&o[2], i * M + j)), T);
+    }
+}
+
+/* 3DCONV (reading #26): 27-point stencil on A[NI][NJ][NK]: the 2DCONV weights on
+ * each (j,k)-plane (C9 index (dk+1)*3 + (dj+1)) scaled by g = (0.25, 0.5, 0.25)
+ * for di = -1, 0, +1; weights formed in fp64 and RNE-rounded to T; products
+ * rounded, summed left to right (di outer, then the 2DCONV order); border +0. */
+static double conv3d_at(int T, const obj_t *A, size_t NJ, size_t NK, size_t i, size_t j, size_t k) {
+  static const double g[3] = {0.25, 0.5, 0.25};
+  double acc = 0.0;
+  int p, q;
+  for (p = 0; p < 3; p++)
+    for (q = 0; q < 9; q++) {
+      const int di = p - 1, dj = (q % 3) - 1, dk = (q / 3) - 1;
+      double w = t_lit(T, g[p] * CONV2D_C[q]);
+      double v = ld(A, ((i + di) * NJ + (j + dj)) * NK + (k + dk));
+      double prod = t_mul(T, w, v);
+      acc = (p == 0 && q == 0) ? prod : t_add(T, acc, prod);
+    }
+  return acc;
+}
+static void app_conv3d(obj_t *o, const int64_t *d) {
+  size_t NI = d[0], NJ = d[1], NK = d[2], i, j, k;
+  int T = W2(o[0].type, o[1].type);
+  for (i = 0; i < NI; i++)
+    for (j = 0; j < NJ; j++)
+      for (k = 0; k < NK; k++) {
+        int border = i == 0 || j == 0 || k == 0 || i + 1 >= NI || j + 1 >= NJ || k + 1 >= NK;
+        st(&o[1], (i * NJ + j) * NK + k, border ? 0.0 : conv3d_at(T, &o[0], NJ, NK, i, j, k), T);
+      }
+}
+
+/* FDTD-2D (reading #27), TMAX steps over ex, ey, hz (NX x NY), each statement a
+ * separate pass in its own compute type:
+ *   ey[0][j] = fict[t]
+ *   ey[i][j] = ey[i][j] - 0.5 (hz[i][j] - hz[i-1][j])            i >= 1
+ *   ex[i][j] = ex[i][j] - 0.5 (hz[i][j] - hz[i][j-1])            j >= 1
+ *   hz[i][j] = hz[i][j] - 0.7 (ex[i][j+1] - ex[i][j] + ey[i+1][j] - ey[i][j])
+ *                                                   i < NX-1, j < NY-1 */
+static void app_fdtd2d(obj_t *o, const int64_t *d) {
+  size_t TM = d[0], NX = d[1], NY = d[2], t, i, j;
+  int T1 = W2(o[0].type, o[2].type), T2 = W2(o[2].type, o[3].type);
+  int T3 = W2(o[1].type, o[3].type), T4 = W3(o[3].type, o[1].type, o[2].type);
+  double h2 = t_lit(T2, 0.5), h3 = t_lit(T3, 0.5), c4 = t_lit(T4, 0.7);
+  for (t = 0; t < TM; t++) {
+    for (j = 0; j < NY; j++) st(&o[2], j, ld(&o[0], t), T1);
+    for (i = 1; i < NX; i++)
+      for (j = 0; j < NY; j++) {
+        double dh = t_sub(T2, ld(&o[3], i * NY + j), ld(&o[3], (i - 1) * NY + j));
+        st(&o[2], i * NY + j, t_sub(T2, ld(&o[2], i * NY + j), t_mul(T2, h2, dh)), T2);
+      }
+    for (i = 0; i < NX; i++)
+      for (j = 1; j < NY; j++) {
+        double dh = t_sub(T3, ld(&o[3], i * NY + j), ld(&o[3], i * NY + j - 1));
+        st(&o[1], i * NY + j, t_sub(T3, ld(&o[1], i * NY + j), t_mul(T3, h3, dh)), T3);
+      }
+    for (i = 0; i + 1 < NX; i++)
+      for (j = 0; j + 1 < NY; j++) {
+        double s = t_sub(T4, ld(&o[1], i * NY + j + 1), ld(&o[1], i * NY + j));
+        s = t_add(T4, s, ld(&o[2], (i + 1) * NY + j));
+        s = t_sub(T4, s, ld(&o[2], i * NY + j));
+        st(&o[3], i * NY + j, t_sub(T4, ld(&o[3], i * NY + j), t_mul(T4, c4, s)), T4);
+      }
+  }
+}
+
 static int run_objects(const app_def_t *a, const int64_t *d, const double *sc, obj_t *o) {
+  if (!strcmp(a->kind, "syr2k")) { app_syr2k(o, d, sc); return 0; }
+  if (!strcmp(a->kind, "conv3d")) { app_conv3d(o, d); return 0; }
+  if (!strcmp(a->kind, "fdtd2d")) { app_fdtd2d(o, d); return 0; }
   if (!strcmp(a->kind, "mvt")) { app_mvt(o, d); return 0; }
   if (!strcmp(a->kind, "syrk")) { app_syrk(o, d, sc); return 0; }
   if (!strcmp(a->kind, "conv2d")) { app_conv2d(o, d); return 0; }
@@ -863,6 +962,32 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
       int border = (i == 0 || j == 0 || i + 1 >= NI || j + 1 >= NJ);
       vals[k] = round_to(prec[1], border ? 0.0 : conv2d_at(T, &in[0], NJ, i, j), T);
     }
+  } else if (!strcmp(kind, "syr2k")) {
+    size_t M = d[1], N = d[0];
+    int T = W3(prec[0], prec[1], prec[2]);
+    double al = t_lit(T, scalar_or(sc, 0, 32412.0)), be = t_lit(T, scalar_or(sc, 1, 2123.0));
+    for (k = 0; k < n; k++) {
+      size_t i = rows[k], j = cols[k];
+      double s1 = dot_chain(T, &in[0], i, M, &in[1], j, M, N);
+      double c1 = round_to(prec[2], t_fma(T, al, s1, t_mul(T, be, ld(&in[2], i * M + j))), T);
+      double s2 = dot_chain(T, &in[1], i, M, &in[0], j, M, N);
+      vals[k] = round_to(prec[2], t_fma(T, al, s2, c1), T);
+    }
+  } else if (!strcmp(kind, "conv3d")) {
+    size_t NI = d[0], NJ = d[1], NK = d[2];
+    int T = W2(prec[0], prec[1]);
+    for (k = 0; k < n; k++) {
+      size_t i = rows[k], j = cols[k] / NK, kk = cols[k] % NK;
+      int border = i == 0 || j == 0 || kk == 0 || i + 1 >= NI || j + 1 >= NJ || kk + 1 >= NK;
+      vals[k] = round_to(prec[1], border ? 0.0 : conv3d_at(T, &in[0], NJ, NK, i, j, kk), T);
+    }
+  } else if (!strcmp(kind, "fdtd2d")) {     /* time-stepped: every entry depends on all */
+    obj_t o[8];
+    const app_def_t *ap;
+    int64_t dd[8];
+    if (run_to_objects(kind, dims, ndims, sc, prec, inputs, o, &ap, dd)) return 1;
+    for (k = 0; k < n; k++) vals[k] = ld(&o[m], (size_t)(rows[k] * C[m] + cols[k]));
+    free_objects(o, ap->nobj);
   } else {                                  /* corr / covar: symmat entries */
     int corr = !strcmp(kind, "corr");
     size_t N = d[0], M = d[1];

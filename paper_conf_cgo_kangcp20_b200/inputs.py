@@ -25,7 +25,7 @@ import numpy as np
 DEFAULT_HI = {
     "gemm": 513.0, "2mm": 2051.0, "3mm": 515.0, "atax": 4094.0,
     "bicg": 4096.0, "gesummv": 4096.0, "corr": 2047.0, "covar": 2048.0,
-    "mvt": 2.0, "syrk": 1026.0, "conv2d": 1.0,
+    "mvt": 2.0, "syrk": 1026.0, "conv2d": 1.0, "syr2k": 2050.0, "conv3d": 59.0, "fdtd2d": 2041.0,
 }
 # BICG's r and p vectors span 0 - 4096*pi (Table 4)
 DEFAULT_HI_OBJECT = {("bicg", "r"): 4096.0 * math.pi, ("bicg", "p"): 4096.0 * math.pi}

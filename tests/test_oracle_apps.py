@@ -53,11 +53,12 @@ def test_object_tables(oracle_lib):
 # ----------------------------------------------------- f64 vs numpy textbook
 DIMS = {"gemm": [13, 17, 11], "2mm": [9, 14, 11, 7], "3mm": [6, 9, 8, 10, 7],
         "atax": [37, 45], "bicg": [41, 33], "gesummv": [29], "corr": [40, 23], "covar": [35, 19],
-        "mvt": [43], "syrk": [31, 18], "conv2d": [17, 23]}
+        "mvt": [43], "syrk": [31, 18], "conv2d": [17, 23], "syr2k": [27, 15], "conv3d": [7, 9, 11],
+        "fdtd2d": [4, 13, 17]}
 CONV2D_C = [0.2, -0.3, 0.4, 0.5, 0.6, 0.7, -0.8, -0.9, 0.10]
 
 
-def numpy_ref(kind, ins, objs, scalars=None):
+def numpy_ref(kind, ins, objs, scalars=None, dims=None):
     A = [None if a is None else a.astype(np.float64).reshape(o["rows"], o["cols"])
          for a, o in zip(ins, objs)]
     if kind == "gemm":
@@ -101,6 +102,27 @@ def numpy_ref(kind, ins, objs, scalars=None):
         for c, x, y in zip(CONV2D_C, di, dj):
             b[1:-1, 1:-1] += c * a[1 + x:ni - 1 + x, 1 + y:nj - 1 + y]
         return {1: b}
+    if kind == "syr2k":
+        al, be = scalars or (32412.0, 2123.0)
+        return {2: al * (A[0].T @ A[1] + A[1].T @ A[0]) + be * A[2]}
+    if kind == "conv3d":
+        ni, nj, nk = dims
+        a = A[0].reshape(ni, nj, nk)
+        b = np.zeros_like(a)
+        for p, g in enumerate((0.25, 0.5, 0.25)):
+            for q, c in enumerate(CONV2D_C):
+                di, dj, dk = p - 1, q % 3 - 1, q // 3 - 1
+                b[1:-1, 1:-1, 1:-1] += g * c * a[1 + di:ni - 1 + di, 1 + dj:nj - 1 + dj, 1 + dk:nk - 1 + dk]
+        return {1: b.reshape(ni, nj * nk)}
+    if kind == "fdtd2d":
+        tmax = objs[0]["cols"]
+        fict, ex, ey, hz = A[0][0].copy(), A[1].copy(), A[2].copy(), A[3].copy()
+        for t in range(tmax):
+            ey[0, :] = fict[t]
+            ey[1:, :] = ey[1:, :] - 0.5 * (hz[1:, :] - hz[:-1, :])
+            ex[:, 1:] = ex[:, 1:] - 0.5 * (hz[:, 1:] - hz[:, :-1])
+            hz[:-1, :-1] = hz[:-1, :-1] - 0.7 * (ex[:-1, 1:] - ex[:-1, :-1] + ey[1:, :-1] - ey[:-1, :-1])
+        return {1: ex, 2: ey, 3: hz}
     raise KeyError(kind)
 
 
@@ -113,7 +135,7 @@ def test_f64_config_matches_numpy(oracle_lib, kind, iset):
     objs = oracle.app_objects(kind, dims)
     ins = gen.make_inputs(kind, objs, iset, seed=3)
     fin = oracle.reference(kind, dims, ins)
-    for m, want in numpy_ref(kind, ins, objs).items():
+    for m, want in numpy_ref(kind, ins, objs, dims=dims).items():
         got = fin[m]
         assert got.dtype == np.float64
         np.testing.assert_allclose(got, want, rtol=1e-12, atol=1e-12 * np.abs(want).max())
@@ -155,7 +177,8 @@ def _fits(v, p):
     return np.all(np.abs(v) <= lim)
 
 
-@pytest.mark.parametrize("kind", ["gemm", "2mm", "3mm", "atax", "bicg", "gesummv", "mvt", "syrk"])
+@pytest.mark.parametrize("kind", ["gemm", "2mm", "3mm", "atax", "bicg", "gesummv", "mvt", "syrk",
+                                  "syr2k"])
 def test_exact_integer_results_every_config(oracle_lib, kind):
     """With small non-negative integer inputs every partial sum is an integer
     bounded by the final value, so every configuration whose objects can hold
@@ -166,10 +189,10 @@ def test_exact_integer_results_every_config(oracle_lib, kind):
     dims = {"atax": [300, 77], "bicg": [270, 93], "gesummv": [75]}.get(kind, DIMS[kind])
     objs = oracle.app_objects(kind, dims)
     ins = _exact_ints(kind, dims, objs, rng)
-    sc = (2.0, 3.0) if kind in ("gemm", "gesummv", "syrk") else None
+    sc = (2.0, 3.0) if kind in ("gemm", "gesummv", "syrk", "syr2k") else None
     if kind == "syrk":        # C must be symmetric for the textbook form to apply
         ins[1] = np.triu(ins[1]) + np.triu(ins[1], 1).T
-    exact = {m: np.rint(v) for m, v in numpy_ref(kind, ins, objs, sc).items()}
+    exact = {m: np.rint(v) for m, v in numpy_ref(kind, ins, objs, sc, dims).items()}
     n_checked = 0
     for prec in itertools.product([F64, F32, F16], repeat=len(objs)):
         if not all(_fits(v, prec[m]) for m, v in exact.items()):

@@ -10,7 +10,8 @@ from paper_conf_cgo_kangcp20_b200 import inputs as gen
 
 CASES = {"gemm": [37, 29, 41], "2mm": [19, 23, 17, 21], "3mm": [11, 13, 9, 15, 10],
          "atax": [300, 77], "bicg": [270, 93], "gesummv": [75], "corr": [60, 17], "covar": [55, 13],
-         "mvt": [301], "syrk": [23, 14], "conv2d": [15, 21]}
+         "mvt": [301], "syrk": [23, 14], "conv2d": [15, 21], "syr2k": [21, 13],
+         "conv3d": [6, 7, 9], "fdtd2d": [3, 11, 13]}
 
 
 @pytest.mark.parametrize("kind", sorted(CASES))
