@@ -82,11 +82,14 @@ static const AppDef kApps[] = {
     {"mvt", 5, 1, {{"A", 0, 0}, {"x1", 2, 1}, {"x2", 2, 1}, {"y1", 0, 0}, {"y2", 0, 0}}},
     {"syrk", 2, 2, {{"A", 0, 0}, {"C", 2, 1}}},
     {"conv2d", 2, 2, {{"A", 0, 0}, {"B", 1, 1}}},
+    {"syr2k", 3, 2, {{"A", 0, 0}, {"B", 0, 0}, {"C", 2, 1}}},
+    {"conv3d", 2, 3, {{"A", 0, 0}, {"B", 1, 1}}},
+    {"fdtd2d", 4, 3, {{"fict", 0, 0}, {"ex", 2, 1}, {"ey", 2, 1}, {"hz", 2, 1}}},
 };
 enum AppKind { K_GEMM, K_2MM, K_3MM, K_ATAX, K_BICG, K_GESUMMV, K_CORR, K_COVAR, K_MVT, K_SYRK,
-               K_CONV2D };
+               K_CONV2D, K_SYR2K, K_CONV3D, K_FDTD2D };
 // statements that read or write each object (for ps_search's object order)
-static const int kTouch[11][8] = {
+static const int kTouch[14][8] = {
     {1, 1, 1},                  // gemm: C <- aAB + bC
     {1, 1, 2, 1, 1},            // 2mm
     {1, 1, 1, 1, 2, 2, 1},      // 3mm
@@ -98,6 +101,9 @@ static const int kTouch[11][8] = {
     {2, 1, 1, 1, 1},            // mvt
     {1, 1},                     // syrk
     {1, 1},                     // conv2d
+    {2, 2, 2},                  // syr2k
+    {1, 1},                     // conv3d
+    {1, 2, 3, 3},               // fdtd2d (per time step)
 };
 
 }  // namespace ps
@@ -239,6 +245,9 @@ void shapes(ps_app *a) {
       break;
     case K_SYRK: set(0, d[0], d[1]); set(1, d[1], d[1]); break;
     case K_CONV2D: set(0, d[0], d[1]); set(1, d[0], d[1]); break;
+    case K_SYR2K: set(0, d[0], d[1]); set(1, d[0], d[1]); set(2, d[1], d[1]); break;
+    case K_CONV3D: set(0, d[0], d[1] * d[2]); set(1, d[0], d[1] * d[2]); break;
+    case K_FDTD2D: set(0, 1, d[0]); set(1, d[1], d[2]); set(2, d[1], d[2]); set(3, d[1], d[2]); break;
   }
 }
 
@@ -389,6 +398,29 @@ ps_status run_statements(Ctx &c) {
     case K_CONV2D:
       S_(conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st));
       break;
+    case K_SYR2K: {   // C <- alpha A^T B + beta C ; C <- alpha B^T A + C
+      const int64_t N = d[0], M = d[1];
+      for (int s2 = 0; s2 < 2; s2++) {
+        const int x = s2 ? 1 : 0, y = s2 ? 0 : 1;
+        GemmArgs g{};
+        g.M = M; g.N = M; g.K = N;
+        g.A = MatDesc{P[x], p[x], 1, M};   // A(i, k) = X[k][i]
+        g.B = MatDesc{P[y], p[y], M, 1};   // B(k, j) = Y[k][j]
+        g.C = P[2]; g.c_type = p[2]; g.ldc = M;
+        g.Cin = P[2]; g.cin_type = p[2];
+        g.epi = EPI_AXPBY; g.alpha = a->sc[0]; g.beta = s2 ? 1.0 : a->sc[1];
+        g.T = compute_type({p[0], p[1], p[2]});
+        S_(contraction(c, g));
+      }
+      break;
+    }
+    case K_CONV3D:
+      S_(conv3d_async(P[0], p[0], P[1], p[1], d[0], d[1], d[2], c.st));
+      break;
+    case K_FDTD2D:
+      for (int64_t t = 0; t < d[0]; t++)
+        S_(fdtd2d_step_async(P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st));
+      break;
   }
 #undef S_
   return PS_OK;
@@ -536,9 +568,12 @@ ps_status ps_app_create(const char *kind, const int64_t *dims, int ndims, const 
   if (k == K_GEMM) { a->sc[0] = 32412.0; a->sc[1] = 2123.0; }
   if (k == K_GESUMMV) { a->sc[0] = 43532.0; a->sc[1] = 12313.0; }
   if (k == K_CORR) { a->sc[0] = 0.005; }
-  if (k == K_SYRK) { a->sc[0] = 32412.0; a->sc[1] = 2123.0; }
+  if (k == K_SYRK || k == K_SYR2K) { a->sc[0] = 32412.0; a->sc[1] = 2123.0; }
   if (scalars) {
-    if (k == K_GEMM || k == K_GESUMMV || k == K_SYRK) { a->sc[0] = scalars[0]; a->sc[1] = scalars[1]; }
+    if (k == K_GEMM || k == K_GESUMMV || k == K_SYRK || k == K_SYR2K) {
+      a->sc[0] = scalars[0];
+      a->sc[1] = scalars[1];
+    }
     if (k == K_CORR) a->sc[0] = scalars[0];
   }
   shapes(a);

@@ -74,6 +74,12 @@ ps_status mvt_async(const void *A, int ta, int64_t n, void *x1, int t1, void *x2
                     const void *y1, int ty1, const void *y2, int ty2, void *partial, cudaStream_t st);
 // 2DCONV 3x3 stencil (reading #24): B_ij = sum of 9 rounded products, left to right; border +0
 ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, cudaStream_t st);
+// 3DCONV 27-point stencil (reading #26) on NI x NJ x NK
+ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
+                       cudaStream_t st);
+// one FDTD-2D time step t (reading #27): ey, ex, hz passes
+ps_status fdtd2d_step_async(const void *fict, int tf, void *ex, int tex, void *ey, int tey, void *hz,
+                            int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st);
 ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
                        int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
                        double eps, void *partial, cudaStream_t st);

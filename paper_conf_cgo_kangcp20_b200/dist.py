@@ -55,6 +55,12 @@ def _statements(kind, d):
         return [("mm", 0, 0, 1, (d[1], d[1], d[0] / 2.0))]
     if kind == "conv2d":
         return [("ew", [0, 1])]
+    if kind == "syr2k":
+        return [("mm", 0, 1, 2, (d[1], d[1], d[0])), ("mm", 1, 0, 2, (d[1], d[1], d[0]))]
+    if kind == "conv3d":
+        return [("ew", [0, 1])]
+    if kind == "fdtd2d":
+        return [("ew", [1, 2, 3])] * int(d[0])
     raise KeyError(kind)
 
 

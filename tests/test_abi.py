@@ -12,7 +12,8 @@ from paper_conf_cgo_kangcp20_b200 import binding as B
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 APPS = {"gemm": [13, 17, 11], "2mm": [9, 14, 11, 7], "3mm": [6, 9, 8, 10, 7],
         "atax": [37, 45], "bicg": [41, 33], "gesummv": [29], "corr": [40, 23], "covar": [35, 19],
-        "mvt": [43], "syrk": [31, 18], "conv2d": [17, 23]}
+        "mvt": [43], "syrk": [31, 18], "conv2d": [17, 23],
+        "syr2k": [27, 15], "conv3d": [7, 9, 11], "fdtd2d": [4, 13, 17]}
 
 
 @pytest.fixture(scope="module")

@@ -104,6 +104,12 @@ SIMT_CASES = [
     ("syrk", [129, 257], "default", None),
     ("conv2d", [200, 300], "random", None),
     ("conv2d", [37, 65], "image", None),
+    ("syr2k", [260, 70], "random", (1.5, 1.2)),
+    ("syr2k", [67, 130], "default", None),
+    ("conv3d", [20, 30, 70], "random", None),
+    ("conv3d", [9, 17, 300], "image", None),
+    ("fdtd2d", [5, 130, 70], "random", None),
+    ("fdtd2d", [20, 33, 301], "default", None),
 ]
 
 

@@ -113,6 +113,27 @@ def test_syrk_app_tc_bound(torch, dims, c_prec):
     assert abs(r["quality"] - ro["quality"]) <= 1e-3
 
 
+@pytest.mark.parametrize("dims,c_prec", [([264, 136], B.F32), ([200, 264], B.F16)])
+def test_syr2k_app_tc_bound(torch, dims, c_prec):
+    """SYR2K app (reading #25): two tcgen05 statements into the same C.  Each
+    statement contributes its gamma_K bound; C is rounded once per statement."""
+    sc = (1.5, 1.2)
+    app, ins, oref = setup(torch, "syr2k", dims, "random", sc)
+    prec = [B.F16, B.F16, c_prec]
+    r = app.run_config(prec)
+    ro, delivered = oracle.evaluate("syr2k", dims, prec, ins, oref, sc)
+    M = dims[1]
+    got = app.outputs[2].cpu().numpy().astype(np.float64).reshape(M, M)
+    want = delivered[2].astype(np.float64).reshape(M, M)
+    st = oracle.run_config("syr2k", dims, prec, ins, sc)
+    a16 = np.abs(st[0].astype(np.float64).reshape(dims[0], M))
+    b16 = np.abs(st[1].astype(np.float64).reshape(dims[0], M))
+    u = ulp(want, np.float16 if c_prec == B.F16 else np.float32)
+    bound = sc[0] * 2 * gamma(dims[0]) * (a16.T @ b16 + b16.T @ a16) * (1 + 2 ** -10) + 4 * u
+    assert np.all(np.abs(got - want) <= bound)
+    assert abs(r["quality"] - ro["quality"]) <= 1e-3
+
+
 @pytest.mark.parametrize("kind,dims", [("2mm", [136, 264, 200, 72]), ("3mm", [136, 72, 200, 64, 128])])
 def test_chain_tc_relative(torch, kind, dims):
     """Every config of the chain apps with tensor cores enabled: fp16 statements
