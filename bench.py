@@ -47,6 +47,9 @@ WORKLOADS = {
     "mvt": [("mvt", [16384])],
     "stencil": [("conv2d", [16384, 16384])],
     "syrk": [("syrk", [8192, 8192])],
+    "syr2k": [("syr2k", [8192, 8192])],
+    "stencil3d": [("conv3d", [512, 512, 512])],
+    "fdtd": [("fdtd2d", [50, 8192, 8192])],
 }
 SIZE = {0: 8, 1: 4, 2: 2}
 # CPU-oracle samples: (reduced dimension, work exponent) -- the oracle needs ~40 s
@@ -54,7 +57,10 @@ SIZE = {0: 8, 1: 4, 2: 2}
 # the reduced size and extrapolate throughput by (N_sample / N)^exponent (O(N^2)
 # mat-vec, O(N^3) contractions); labelled "extrapolated" in the JSON.
 CPU_SAMPLE = {"matvec": (8192, 2), "gemm64": (None, 0), "contract": (384, 3), "contract3mm": (256, 3),
-              "corr": (512, 3), "mvt": (8192, 2), "stencil": (4096, 2), "syrk": (512, 3)}
+              "corr": (512, 3), "mvt": (8192, 2), "stencil": (4096, 2), "syrk": (512, 3),
+              "syr2k": (384, 3), "stencil3d": (128, 3), "fdtd": (None, 0)}
+# per-dimension sample overrides (the exponent then counts the scaled dimensions)
+CPU_SAMPLE_DIMS = {"fdtd": [50, 1024, 1024]}
 
 
 def log(*a):
@@ -133,11 +139,22 @@ def kernel_bytes(kind, dims, prec):
                                             SIZE[prec[4]])
     if kind == "conv2d":   # A read once, B written once
         return dims[0] * dims[1] * (SIZE[prec[0]] + SIZE[prec[1]])
+    if kind == "conv3d":
+        return dims[0] * dims[1] * dims[2] * (SIZE[prec[0]] + SIZE[prec[1]])
+    if kind == "fdtd2d":   # per step: ey rd+wr, hz rd | ex rd+wr, hz rd | ex, ey rd, hz rd+wr
+        return dims[0] * (dims[1] * dims[2] * (3 * SIZE[prec[1]] + 3 * SIZE[prec[2]] + 4 * SIZE[prec[3]]) +
+                          dims[2] * SIZE[prec[2]])
     return None
 
 
 # contraction statements: (a, b, out, M, N, K-flop-factor); SYRK computes the
 # upper triangle only, so its algorithmic work is M*M*N multiply-adds / 2 * 2.
+A3_KERNELS = {"atax": "tile_kernel + finalizers", "bicg": "tile_kernel + finalizers",
+              "gesummv": "tile_kernel + finalizers + axpby", "mvt": "mvt tile_kernel + finalizers",
+              "conv2d": "conv2d_kernel", "conv3d": "conv3d_kernel",
+              "fdtd2d": "fdtd_ey/ex/hz_kernel x TMAX"}
+
+
 def _contractions(kind, d):
     if kind == "gemm":
         return [(0, 1, 2, d[0], d[1], d[2])]
@@ -149,6 +166,8 @@ def _contractions(kind, d):
         return [(0, 0, 3 if kind == "corr" else 2, d[1], d[1], d[0] / 2.0)]
     if kind == "syrk":
         return [(0, 0, 1, d[1], d[1], d[0] / 2.0)]
+    if kind == "syr2k":
+        return [(0, 1, 2, d[1], d[1], d[0]), (1, 0, 2, d[1], d[1], d[0])]
     return []
 
 
@@ -187,6 +206,46 @@ def contraction_roofline(apps, last):
             "statements_by_path": paths}
 
 
+# FP ops per output of the ALU-heavy stencils (products rounded separately, R4):
+# 3DCONV 27 multiplies + 26 adds (reading #26)
+STENCIL_OPS = {"conv3d": 53}
+
+
+def stencil_roofline(apps, last, hbm):
+    """a3 of 3DCONV: per configuration the ideal time is max(ALU time, HBM time) with
+    ALU peak = FP32 (128) or FP64 (64) lanes/clk/SM x 148 SMs x 1965 MHz (one lane-op
+    per FMUL/FADD) and HBM = the measured copy bandwidth; frac = sum ideal / sum measured."""
+    lanes = {1: 148 * 128 * 1.965e9, 0: 148 * 64 * 1.965e9}
+    ideal = meas = ops = 0.0
+    bound_t = {"alu": 0.0, "hbm": 0.0}
+    for a in apps:
+        k = a["kind"]
+        if k not in STENCIL_OPS:
+            return None
+        m = a["app"].num_objects
+        n_out = float(np.prod(a["dims"]))
+        for r in last[k]:
+            p = decode(int(r["config_id"]), m)
+            T = 0 if 0 in p else 1
+            t_alu = n_out * STENCIL_OPS[k] / lanes[T]
+            t_hbm = kernel_bytes(k, a["dims"], p) / (hbm * 1e9)
+            ideal += max(t_alu, t_hbm)
+            bound_t["alu" if t_alu >= t_hbm else "hbm"] += max(t_alu, t_hbm)
+            ops += n_out * STENCIL_OPS[k]
+            meas += float(r["kernel_ms"]) * 1e-3
+    if meas <= 0:
+        return None
+    return {"bound": max(bound_t, key=bound_t.get), "achieved": round(ops / meas / 1e12, 3),
+            "unit": "TFLOP/s (FP32/FP64 lane-ops)", "peak": {"fp32": round(lanes[1] / 1e12, 1),
+                                                              "fp64": round(lanes[0] / 1e12, 1),
+                                                              "hbm_gbs": hbm},
+            "frac": round(ideal / meas, 4), "traffic": None,
+            "peak_source": "ALU peaks derived from unit counts (B200_PROFILING.md: 148 SMs, 1965 MHz); "
+                           "HBM = MEASURED_PEAKS.json; ideal per config = max(ALU, HBM) time",
+            "kernel": "a3 conv3d_kernel (2.5-D smem blocking, cp.async ring)",
+            "ideal_time_share": {k2: round(v / ideal, 4) for k2, v in bound_t.items()}}
+
+
 def convert_bytes(objects, prec):
     b = 0
     for o, p in zip(objects, prec):
@@ -207,6 +266,10 @@ def decode(cid, m):
 def _sample(workload):
     kind, dims = WORKLOADS[workload][0]
     n_s, expo = CPU_SAMPLE[workload]
+    if workload in CPU_SAMPLE_DIMS:
+        sdims = CPU_SAMPLE_DIMS[workload]
+        factor = float(np.prod(sdims)) / float(np.prod(dims))
+        return kind, dims, sdims, factor, 1
     sdims = dims if n_s is None else [n_s] * len(dims)
     factor = 1.0 if n_s is None else (n_s / float(dims[0])) ** expo
     return kind, dims, sdims, factor, expo
@@ -307,28 +370,35 @@ def whole_program(torch, B, apps, args):
 
 
 # ------------------------------------------------------------ conversion
-def conversion_sweep(torch, B, flush, reps=10):
+def conversion_sweep(torch, B, flush, reps=20, sizes=None):
+    """BASELINE configs[1] / SURVEY §8(d)-2 row 2: source sizes 2^20 .. 2^32 bytes, four
+    directions, L2 flushed before every rep, median of `reps` CUDA-event timings.
+    Algorithmic GB/s = n (s_src + s_dst) / t."""
+    sizes = sizes or [1 << k for k in range(20, 33)]
     out = {}
     TD = {0: torch.float64, 1: torch.float32, 2: torch.float16}
     for st, dt, name in [(1, 2, "f32->f16"), (2, 1, "f16->f32"), (0, 2, "f64->f16"),
                          (0, 1, "f64->f32")]:
-        n = (1 << 30) // SIZE[st]           # 1 GiB source
-        src = torch.zeros(n, dtype=TD[st], device="cuda")
-        dst = torch.empty(n, dtype=TD[dt], device="cuda")
-        for _ in range(3):
-            B.ps_convert(src, st, dst, dt)
-        ts = []
-        for _ in range(reps):
-            flush.zero_()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            B.ps_convert(src, st, dst, dt)
-            e1.record()
-            torch.cuda.synchronize()
-            ts.append(e0.elapsed_time(e1))
-        t = float(np.median(ts))
-        out[name] = round(n * (SIZE[st] + SIZE[dt]) / (t * 1e-3) / 1e9, 1)
-        del src, dst
+        row = {}
+        for nbytes in sizes:
+            n = nbytes // SIZE[st]
+            src = torch.zeros(n, dtype=TD[st], device="cuda")
+            dst = torch.empty(n, dtype=TD[dt], device="cuda")
+            for _ in range(3):
+                B.ps_convert(src, st, dst, dt)
+            ts = []
+            for _ in range(reps):
+                flush.zero_()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                B.ps_convert(src, st, dst, dt)
+                e1.record()
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            t = float(np.median(ts))
+            row[nbytes] = round(n * (SIZE[st] + SIZE[dt]) / (t * 1e-3) / 1e9, 1)
+            del src, dst
+        out[name] = row
     return out
 
 
@@ -395,6 +465,7 @@ def main():
         log("rank %d setup %s %s: %d/%d configs, %.1f s" % (rank, kind, dims, len(mine),
                                                               app.space, time.time() - t0))
     total_configs = sum(a["space"] for a in apps)
+    max_obj = max(o["n"] * 4 for a in apps for o in a["app"].objects)
 
     def step(collect=None):
         for a in apps:
@@ -539,15 +610,18 @@ def main():
 
     n_conv_groups = sum(1 for a in apps for r in last[a["kind"]]
                         if convert_bytes(a["app"].objects, decode(int(r["config_id"]), a["app"].num_objects)))
+    knames = sorted({A3_KERNELS.get(a["kind"], a["kind"]) for a in apps})
     roof_a3 = hbm_roof(kb, kt, n_kernel_groups,
-                       "a3 mat-vec statement kernels of one configuration (tile_kernel + finalizers)",
-                       "ratio")
+                       "a3 statement kernels of one configuration (%s)" % ", ".join(knames), "ratio")
     roof_a2 = hbm_roof(cb, ct, n_conv_groups,
                        "a2 conversion kernels of one configuration (convert_kernel)", "convert_ratio")
     roof_mm = contraction_roofline(apps, last) if kb == 0 else None
+    roof_st = stencil_roofline(apps, last, hbm)
     # the dominant phase's kernel is THE roofline; the other is reported beside it
     if roof_mm is not None:
         roof, conv_roof = roof_mm, roof_a2
+    elif roof_st is not None:
+        roof, conv_roof = roof_st, roof_a3
     elif phase["convert"] > phase["kernel"] and roof_a2 is not None:
         roof, conv_roof = roof_a2, roof_a3
     else:
@@ -564,9 +638,12 @@ def main():
     conv = None
     if not args.no_conversion:
         flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
-        conv = conversion_sweep(torch, B, flush)
-        conv = {k: {"gbs": v, "frac_of_measured": round(v / hbm, 4), "frac_of_8tbs": round(v / 8000, 4)}
-                for k, v in conv.items()}
+        sweep = conversion_sweep(torch, B, flush)
+        conv = {k: {"gbs": v[1 << 30], "frac_of_measured": round(v[1 << 30] / hbm, 4),
+                    "frac_of_8tbs": round(v[1 << 30] / 8000, 4),
+                    "min_frac_at_ge_256MB": round(min(g for b, g in v.items() if b >= 256 << 20) / hbm, 4),
+                    "sweep_gbs_by_src_bytes": {str(b): g for b, g in v.items()}}
+                for k, v in sweep.items()}
 
     tot_phase = sum(phase.values())
     line = {
@@ -579,7 +656,8 @@ def main():
                    "apps": ["%s %s" % (a["kind"], "x".join(map(str, a["dims"]))) for a in apps],
                    "configs_per_step": total_configs, "input_set": args.input_set, "toq": args.toq,
                    "step": "a0 reference + full 3^M config space per app (a1-a7)",
-                   "l2": "inputs larger than L2 (each matrix 1 GiB fp32 > 126 MB)",
+                   "l2": "inputs larger than L2: largest object %.0f MB at fp32 vs 126 MB L2%s" % (
+                       max_obj / 1e6, "" if max_obj > 126e6 else " (NOT larger: launch-bound case)"),
                    "parallelism": "configs partitioned over %d GPU(s), NCCL result gather" % world},
         "e2e": e2e, "gpu_launches": launches,
         "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
