@@ -354,7 +354,7 @@ def whole_program(torch, B, apps, args):
         app = a["app"]
         host = [torch.from_numpy(x.reshape(-1)).pin_memory() if x is not None else None for x in a["ins"]]
         m = app.num_objects
-        res = D.decide(app, host, db, toq=args.toq)
+        res = D.decide(app, host, db, toq=args.toq, reps=3)
         orig = [app.run_config_host([1] * m, host, [0] * m, toq=args.toq)["total_ms"] for _ in range(3)]
         mine = [app.run_config_host(res["prec"], host, res["methods"], toq=args.toq)["total_ms"]
                 for _ in range(3)]

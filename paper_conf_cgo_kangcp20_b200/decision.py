@@ -100,9 +100,12 @@ def best_method(db: dict, n: int, target: int, intermediates=(B.F32,)):
 
 
 # ------------------------------------------------------------ decision maker
-def decide(app, host_inputs, db: dict, toq: float = 0.9, threads: int = 0, verify: bool = True):
+def decide(app, host_inputs, db: dict, toq: float = 0.9, threads: int = 0, verify: bool = True,
+           reps: int = 1):
     """Alg. 1 over all objects with PFP initialisation.  Returns a dict with the chosen
-    precisions and methods, the final measured run, and the trial log."""
+    precisions and methods, the final measured run, and the trial log.  ``reps`` > 1
+    times every trial that many times and keeps the median total (the quality of a
+    configuration is deterministic), so that timing noise cannot flip a choice."""
     objs = app.objects
     M = app.num_objects
     inputs = [k for k, o in enumerate(objs) if o["role"] in (0, 2)]
@@ -120,7 +123,10 @@ def decide(app, host_inputs, db: dict, toq: float = 0.9, threads: int = 0, verif
     def run_app(prec, meth):                      # Alg. 1 line 8
         key = (tuple(prec), tuple(meth))
         if key not in cache:
-            r = app.run_config_host(prec, host_inputs, meth, threads=threads, toq=toq)
+            runs = [app.run_config_host(prec, host_inputs, meth, threads=threads, toq=toq)
+                    for _ in range(max(1, reps))]
+            runs.sort(key=lambda x: x["total_ms"])
+            r = runs[len(runs) // 2]
             r["kernel_side_ms"] = r["total_ms"] - r["transfer_ms"]
             cache[key] = r
             log.append({"prec": list(prec), "methods": list(meth), "total_ms": r["total_ms"],
