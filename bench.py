@@ -457,7 +457,7 @@ def main():
         ins = gen.make_inputs(kind, app.objects, args.input_set)
         dins = [torch.from_numpy(a.reshape(-1)).cuda() if a is not None else None for a in ins]
         app.bind(dins)
-        refs = app.reference()
+        refs = D.sharded_reference(app, world, rank)
         ids = list(range(app.space))
         mine = D.partition_configs(kind, dims, app.objects, ids, world, rank) if world > 1 else ids
         apps.append(dict(kind=kind, dims=dims, app=app, ins=ins, refs=refs, ids=mine,
@@ -469,7 +469,7 @@ def main():
 
     def step(collect=None):
         for a in apps:
-            a["app"].reference(refs=a["refs"])                       # a0
+            D.sharded_reference(a["app"], world, rank, refs=a["refs"])   # a0 (row-sharded)
             arr, _ = a["app"].sweep_raw(a["ids"], args.toq)          # a1-a7 (local share)
             if world > 1:
                 arr = D.gather_results(arr)                          # NCCL gather
@@ -524,7 +524,7 @@ def main():
         def step_e2e():
             for a, hin in zip(apps, host):
                 a["app"].load_host(hin)                               # H2D of the inputs
-                a["app"].reference(refs=a["refs"])
+                D.sharded_reference(a["app"], world, rank, refs=a["refs"])
                 arr, _ = a["app"].sweep_raw(a["ids"], args.toq)       # results read back (D2H)
                 if world > 1:
                     D.gather_results(arr)

@@ -133,6 +133,34 @@ PS_API ps_status ps_app_reference(ps_app *app, double *const *ref_outputs, void 
 /* Use externally computed fp64 reference outputs instead (e.g. gathered). */
 PS_API ps_status ps_app_set_reference(ps_app *app, const double *const *ref_outputs);
 
+/* a0 sharded by contiguous output rows (north star item 5): the
+ * contraction apps (GEMM, 2MM, 3MM, SYRK, SYR2K, CORR, COVAR) have one scored
+ * output whose rows can be computed independently.
+ *   ps_app_shard_rows:       that output's row count; 0 = the app is not
+ *                            row-shardable (mat-vec / stencil references are one
+ *                            streaming pass: every rank runs ps_app_reference).
+ *   ps_app_shard_triangular: 1 when row i costs ~ (rows - i) (upper tiles + mirror:
+ *                            SYRK, CORR, COVAR) so callers can balance the split.
+ *   ps_app_reference_rows:   rows [row0, row1) of the all-f64 run written into
+ *                            ref_outputs[m] at their full-matrix offsets
+ *                            (ref_outputs[m]: caller-owned device, n elements);
+ *                            every element of those rows is bit-identical to
+ *                            ps_app_reference, except the strictly-lower part of
+ *                            triangular outputs, which is left unspecified.
+ *                            Other rows are not touched.  Synchronises `stream`.
+ *   ps_app_reference_merge:  after the caller has assembled every row (e.g. an
+ *                            NCCL all-gather), mirror the upper triangle (and the
+ *                            unit diagonal of CORR) and adopt ref_outputs as the
+ *                            quality reference -- afterwards identical, bit for
+ *                            bit, to ps_app_reference.
+ * Errors: PS_ERR_UNSUPPORTED for non-shardable apps; PS_ERR_INVALID for a row
+ * range outside [0, rows) or a missing buffer; PS_ERR_WORKSPACE if not bound. */
+PS_API int64_t ps_app_shard_rows(const ps_app *app);
+PS_API int ps_app_shard_triangular(const ps_app *app);
+PS_API ps_status ps_app_reference_rows(ps_app *app, int64_t row0, int64_t row1, double *const *ref_outputs,
+                                void *stream);
+PS_API ps_status ps_app_reference_merge(ps_app *app, double *const *ref_outputs, void *stream);
+
 /* ------------------------------------------------------------------------- */
 /* (4) Evaluate one configuration (the hot path).                              */
 typedef struct {

@@ -29,7 +29,8 @@ SYMBOLS = [
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
     "ps_run_config", "ps_sweep", "ps_search", "ps_host_convert", "ps_run_config_host",
-    "ps_transfer",
+    "ps_transfer", "ps_app_shard_rows", "ps_app_shard_triangular", "ps_app_reference_rows",
+    "ps_app_reference_merge",
 ]
 # type-conversion methods for host inputs (Fig. 3)
 XFER_DEVICE, XFER_HOST_LOOP, XFER_HOST_SIMD, XFER_PIPELINE, XFER_TRANSIENT = 0, 1, 2, 3, 4
@@ -107,6 +108,11 @@ def lib():
                 "ps_app_load_host": (ctypes.c_int, [vp, ctypes.POINTER(vp), vp]),
                 "ps_app_reference": (ctypes.c_int, [vp, ctypes.POINTER(vp), vp]),
                 "ps_app_set_reference": (ctypes.c_int, [vp, ctypes.POINTER(vp)]),
+                "ps_app_shard_rows": (ctypes.c_int64, [vp]),
+                "ps_app_shard_triangular": (ctypes.c_int, [vp]),
+                "ps_app_reference_rows": (ctypes.c_int, [vp, ctypes.c_int64, ctypes.c_int64,
+                                                         ctypes.POINTER(vp), vp]),
+                "ps_app_reference_merge": (ctypes.c_int, [vp, ctypes.POINTER(vp), vp]),
                 "ps_config_encode": (ctypes.c_int, [vp, ctypes.POINTER(ctypes.c_int),
                                                     ctypes.POINTER(ctypes.c_uint64)]),
                 "ps_config_decode": (ctypes.c_int, [vp, ctypes.c_uint64, ctypes.POINTER(ctypes.c_int)]),
@@ -287,6 +293,35 @@ class App:
         arr = (vp * self.num_objects)(*[_ptr(t) for t in refs])
         _check(lib().ps_app_reference(self._h, arr, _stream(stream)), "ps_app_reference")
         self.ref = refs
+        return refs
+
+    @property
+    def shard_rows(self) -> int:
+        """Rows of the output a reference shard computes (0: not row-shardable)."""
+        return int(lib().ps_app_shard_rows(self._h))
+
+    @property
+    def shard_triangular(self) -> bool:
+        return bool(lib().ps_app_shard_triangular(self._h))
+
+    def alloc_refs(self):
+        import torch
+        dev = self.workspace.device
+        return [torch.empty(o["n"], dtype=torch.float64, device=dev) if o["is_output"] else None
+                for o in self.objects]
+
+    def reference_rows(self, row0: int, row1: int, refs, stream=None):
+        """ps_app_reference_rows: rows [row0, row1) of the fp64 reference into refs."""
+        arr = (vp * self.num_objects)(*[_ptr(t) for t in refs])
+        _check(lib().ps_app_reference_rows(self._h, int(row0), int(row1), arr, _stream(stream)),
+               "ps_app_reference_rows")
+        return refs
+
+    def reference_merge(self, refs, stream=None):
+        """ps_app_reference_merge: mirror (triangular outputs) and adopt refs."""
+        arr = (vp * self.num_objects)(*[_ptr(t) for t in refs])
+        _check(lib().ps_app_reference_merge(self._h, arr, _stream(stream)), "ps_app_reference_merge")
+        self.ref = list(refs)
         return refs
 
     def set_reference(self, refs):

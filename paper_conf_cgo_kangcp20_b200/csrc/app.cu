@@ -284,42 +284,56 @@ struct Ctx {
   const int *prec;
   void *ptr[8];
   cudaStream_t st;
+  // row-sharded reference: only rows [r0, r1) of the scored output of a
+  // contraction app are computed (r1 < 0: all rows); syrk-like outputs skip the mirror
+  int64_t r0 = 0, r1 = -1;
+  bool sharded() const { return r1 >= 0; }
 };
+
+inline void *eoff(const void *p, int type, int64_t n) {
+  return (char *)p + n * (int64_t)dtype_size(type);
+}
 
 ps_status contraction(Ctx &c, GemmArgs g) {
   const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && g.A.type == PS_F16 &&
-                  g.B.type == PS_F16 && g.T == PS_F32 && gemm_tc_supported(g);
+                  g.B.type == PS_F16 && g.T == PS_F32 && g.row_off == 0 && gemm_tc_supported(g);
   return tc ? gemm_tc_async(g, c.st) : gemm_simt_async(g, c.st);
 }
 
-// out(M x N, row-major) = X(M x K, row-major) . Y(K x N, row-major), R3
-ps_status matmul(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_t K) {
+// out(M x N, row-major) = X(M x K, row-major) . Y(K x N, row-major), R3;
+// rows: restrict to the shard's output rows (X and out row-sliced)
+ps_status matmul(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_t K, bool rows = false) {
+  const int64_t r0 = rows && c.sharded() ? c.r0 : 0;
   GemmArgs g{};
-  g.M = M; g.N = N; g.K = K;
-  g.A = MatDesc{c.ptr[x], c.prec[x], K, 1};
+  g.M = rows && c.sharded() ? c.r1 - c.r0 : M; g.N = N; g.K = K;
+  g.A = MatDesc{eoff(c.ptr[x], c.prec[x], r0 * K), c.prec[x], K, 1};
   g.B = MatDesc{c.ptr[y], c.prec[y], N, 1};
-  g.C = c.ptr[out]; g.c_type = c.prec[out]; g.ldc = N;
+  g.C = eoff(c.ptr[out], c.prec[out], r0 * N); g.c_type = c.prec[out]; g.ldc = N;
   g.epi = EPI_PLAIN;
   g.T = compute_type({c.prec[x], c.prec[y], c.prec[out]});
-  return contraction(c, g);
+  return g.M > 0 ? contraction(c, g) : PS_OK;
 }
 
-// symmat(M x M) = data^T data over N rows, upper tiles + mirror (R3)
+// symmat(M x M) = data^T data over N rows, upper tiles + mirror (R3).  Sharded: the
+// upper part of rows [r0, r1) only; the mirror runs after the gather (reference_merge)
 ps_status syrk(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double div, int diag_one) {
+  const int64_t r0 = c.sharded() ? c.r0 : 0;
   GemmArgs g{};
-  g.M = M; g.N = M; g.K = N;
-  g.A = MatDesc{c.ptr[data], c.prec[data], 1, M};   // A(j1, i) = data[i][j1]
-  g.B = MatDesc{c.ptr[data], c.prec[data], M, 1};   // B(i, j2) = data[i][j2]
-  g.C = c.ptr[sym]; g.c_type = c.prec[sym]; g.ldc = M;
+  g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
+  g.A = MatDesc{eoff(c.ptr[data], c.prec[data], r0), c.prec[data], 1, M};   // A(j1, i) = data[i][j1]
+  g.B = MatDesc{c.ptr[data], c.prec[data], M, 1};                          // B(i, j2) = data[i][j2]
+  g.C = eoff(c.ptr[sym], c.prec[sym], r0 * M); g.c_type = c.prec[sym]; g.ldc = M;
   g.epi = epi; g.div = div;
   if (epi == EPI_AXPBY) {   // SYRK app: C <- alpha data^T data + beta C (C read in place)
-    g.Cin = c.ptr[sym]; g.cin_type = c.prec[sym];
+    g.Cin = g.C; g.cin_type = c.prec[sym];
     g.alpha = c.a->sc[0]; g.beta = c.a->sc[1];
   }
   g.upper_only = 1;
+  g.row_off = r0;
   g.T = compute_type({c.prec[data], c.prec[sym]});
+  if (g.M <= 0) return PS_OK;
   ps_status s = contraction(c, g);
-  if (s != PS_OK) return s;
+  if (s != PS_OK || c.sharded()) return s;
   return mirror_async(c.ptr[sym], c.prec[sym], M, diag_one, c.st);
 }
 
@@ -336,25 +350,26 @@ ps_status run_statements(Ctx &c) {
   } while (0)
   switch (a->kind) {
     case K_GEMM: {   // C <- alpha (A.B) + beta C
+      const int64_t r0 = c.sharded() ? c.r0 : 0;
       GemmArgs g{};
-      g.M = d[0]; g.N = d[1]; g.K = d[2];
-      g.A = MatDesc{P[0], p[0], d[2], 1};
+      g.M = c.sharded() ? c.r1 - c.r0 : d[0]; g.N = d[1]; g.K = d[2];
+      g.A = MatDesc{eoff(P[0], p[0], r0 * d[2]), p[0], d[2], 1};
       g.B = MatDesc{P[1], p[1], d[1], 1};
-      g.C = P[2]; g.c_type = p[2]; g.ldc = d[1];
-      g.Cin = P[2]; g.cin_type = p[2];
+      g.C = eoff(P[2], p[2], r0 * d[1]); g.c_type = p[2]; g.ldc = d[1];
+      g.Cin = g.C; g.cin_type = p[2];
       g.epi = EPI_AXPBY; g.alpha = a->sc[0]; g.beta = a->sc[1];
       g.T = compute_type({p[0], p[1], p[2]});
-      S_(contraction(c, g));
+      if (g.M > 0) S_(contraction(c, g));
       break;
     }
     case K_2MM:
-      S_(matmul(c, 0, 1, 2, d[0], d[1], d[2]));   // C <- A.B
-      S_(matmul(c, 2, 3, 4, d[0], d[3], d[1]));   // E <- C.D
+      S_(matmul(c, 0, 1, 2, d[0], d[1], d[2], true));   // C <- A.B   (rows of E need rows of C)
+      S_(matmul(c, 2, 3, 4, d[0], d[3], d[1], true));   // E <- C.D
       break;
     case K_3MM:
-      S_(matmul(c, 0, 1, 4, d[0], d[1], d[2]));   // E <- A.B
-      S_(matmul(c, 2, 3, 5, d[1], d[3], d[4]));   // F <- C.D
-      S_(matmul(c, 4, 5, 6, d[0], d[3], d[1]));   // G <- E.F
+      S_(matmul(c, 0, 1, 4, d[0], d[1], d[2], true));   // E <- A.B   (rows of G need rows of E)
+      S_(matmul(c, 2, 3, 5, d[1], d[3], d[4]));         // F <- C.D   (every row of F)
+      S_(matmul(c, 4, 5, 6, d[0], d[3], d[1], true));   // G <- E.F
       break;
     case K_ATAX:   // tmp <- A x ; y <- A^T tmp
       S_(rowdot_async(P[0], p[0], d[1], P[1], p[1], P[3], p[3], d[0], d[1], partial, c.st));
@@ -399,18 +414,18 @@ ps_status run_statements(Ctx &c) {
       S_(conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st));
       break;
     case K_SYR2K: {   // C <- alpha A^T B + beta C ; C <- alpha B^T A + C
-      const int64_t N = d[0], M = d[1];
+      const int64_t N = d[0], M = d[1], r0 = c.sharded() ? c.r0 : 0;
       for (int s2 = 0; s2 < 2; s2++) {
         const int x = s2 ? 1 : 0, y = s2 ? 0 : 1;
         GemmArgs g{};
-        g.M = M; g.N = M; g.K = N;
-        g.A = MatDesc{P[x], p[x], 1, M};   // A(i, k) = X[k][i]
-        g.B = MatDesc{P[y], p[y], M, 1};   // B(k, j) = Y[k][j]
-        g.C = P[2]; g.c_type = p[2]; g.ldc = M;
-        g.Cin = P[2]; g.cin_type = p[2];
+        g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
+        g.A = MatDesc{eoff(P[x], p[x], r0), p[x], 1, M};   // A(i, k) = X[k][i]
+        g.B = MatDesc{P[y], p[y], M, 1};                   // B(k, j) = Y[k][j]
+        g.C = eoff(P[2], p[2], r0 * M); g.c_type = p[2]; g.ldc = M;
+        g.Cin = g.C; g.cin_type = p[2];
         g.epi = EPI_AXPBY; g.alpha = a->sc[0]; g.beta = s2 ? 1.0 : a->sc[1];
         g.T = compute_type({p[0], p[1], p[2]});
-        S_(contraction(c, g));
+        if (g.M > 0) S_(contraction(c, g));
       }
       break;
     }
@@ -450,10 +465,13 @@ ps_status ensure_events(ps_app *a, size_t n) {
   return PS_OK;
 }
 
-// a2 .. a5 for one configuration; events ev[0..4] (nullptr = untimed)
+// a2 .. a5 for one configuration; events ev[0..4] (nullptr = untimed); r1 >= 0: only
+// rows [r0, r1) of the scored output (row-sharded reference, no quality)
 ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res,
-                         cudaEvent_t *ev, bool quality) {
+                         cudaEvent_t *ev, bool quality, int64_t r0 = 0, int64_t r1 = -1) {
   Ctx c{a, prec, {nullptr}, st};
+  c.r0 = r0;
+  c.r1 = r1;
   if (ev) PS_CUDA(cudaEventRecord(ev[0], st));
   for (int m = 0; m < a->def->nobj; m++) {
     c.ptr[m] = a->ws + a->slot_off[m];
@@ -514,6 +532,24 @@ float ms_between(cudaEvent_t x, cudaEvent_t y) {
   float t = 0.f;
   if (cudaEventElapsedTime(&t, x, y) != cudaSuccess) return NAN;
   return t;
+}
+
+// the scored output whose rows a reference shard computes (-1: not shardable; the
+// mat-vec and stencil references are single streaming passes, cheaper than a gather)
+int shard_object(const ps_app *a) {
+  switch (a->kind) {
+    case K_GEMM: return 2;
+    case K_2MM: return 4;
+    case K_3MM: return 6;
+    case K_SYRK: return 1;
+    case K_SYR2K: return 2;
+    case K_CORR: return 3;
+    case K_COVAR: return 2;
+    default: return -1;
+  }
+}
+bool shard_triangular(const ps_app *a) {   // upper tiles + mirror: row i costs ~ (rows - i)
+  return a->kind == K_SYRK || a->kind == K_CORR || a->kind == K_COVAR;
 }
 
 ps_status ready(const ps_app *a) {
@@ -656,6 +692,53 @@ ps_status ps_app_reference(ps_app *a, double *const *ref, void *stream) {
     a->ref[m] = ref[m];
   }
   PS_CUDA(cudaStreamSynchronize(st));
+  a->has_ref = true;
+  return PS_OK;
+}
+
+int64_t ps_app_shard_rows(const ps_app *a) {
+  if (!a) return 0;
+  const int m = shard_object(a);
+  return m < 0 ? 0 : a->rows[m];
+}
+
+int ps_app_shard_triangular(const ps_app *a) { return a && shard_object(a) >= 0 && shard_triangular(a); }
+
+ps_status ps_app_reference_rows(ps_app *a, int64_t row0, int64_t row1, double *const *ref, void *stream) {
+  if (!a || !ref) { set_error("ps_app_reference_rows: null pointer"); return PS_ERR_INVALID; }
+  if (!a->bound) { set_error("ps_app_reference_rows: app not bound"); return PS_ERR_WORKSPACE; }
+  const int m = shard_object(a);
+  if (m < 0) { set_error("ps_app_reference_rows: %s is not row-shardable", a->def->kind); return PS_ERR_UNSUPPORTED; }
+  if (row0 < 0 || row1 < row0 || row1 > a->rows[m]) {
+    set_error("ps_app_reference_rows: rows [%lld, %lld) outside [0, %lld)", (long long)row0,
+              (long long)row1, (long long)a->rows[m]);
+    return PS_ERR_INVALID;
+  }
+  if (!ref[m]) { set_error("ps_app_reference_rows: ref %d missing", m); return PS_ERR_INVALID; }
+  cudaStream_t st = (cudaStream_t)stream;
+  int prec[8] = {0};   // all f64 = configuration id 0
+  ps_status s = enqueue_config(a, prec, st, nullptr, nullptr, false, row0, row1);
+  if (s != PS_OK) return s;
+  const int64_t cols = a->cols[m];
+  if (row1 > row0)
+    PS_CUDA(cudaMemcpyAsync(ref[m] + row0 * cols, (const double *)(a->ws + a->slot_off[m]) + row0 * cols,
+                            (size_t)((row1 - row0) * cols) * 8, cudaMemcpyDeviceToDevice, st));
+  PS_CUDA(cudaStreamSynchronize(st));
+  return PS_OK;
+}
+
+ps_status ps_app_reference_merge(ps_app *a, double *const *ref, void *stream) {
+  if (!a || !ref) { set_error("ps_app_reference_merge: null pointer"); return PS_ERR_INVALID; }
+  const int m = shard_object(a);
+  if (m < 0) { set_error("ps_app_reference_merge: %s is not row-shardable", a->def->kind); return PS_ERR_UNSUPPORTED; }
+  if (!ref[m]) { set_error("ps_app_reference_merge: ref %d missing", m); return PS_ERR_INVALID; }
+  cudaStream_t st = (cudaStream_t)stream;
+  if (shard_triangular(a)) {
+    ps_status s = mirror_async(ref[m], PS_F64, a->rows[m], a->kind == K_CORR ? 1 : 0, st);
+    if (s != PS_OK) return s;
+  }
+  PS_CUDA(cudaStreamSynchronize(st));
+  a->ref[m] = ref[m];
   a->has_ref = true;
   return PS_OK;
 }

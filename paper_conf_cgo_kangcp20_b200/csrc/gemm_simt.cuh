@@ -36,6 +36,7 @@ struct Params {
   int tcin;
   int epi;
   int upper_only;
+  int64_t row_off;    // global row of C's row 0 (upper_only test)
   int a_vec, b_vec;   // 16-byte aligned base and leading dimension
 };
 
@@ -93,7 +94,7 @@ __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta
 
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
   const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
-  if (p.upper_only && m0 >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
+  if (p.upper_only && m0 + p.row_off >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
 
   // this thread's contiguous run in the A and B tiles
   const int ea = tid * EA;
@@ -206,7 +207,7 @@ inline Params make_params(const GemmArgs &g) {
   p.B = g.B.p; p.b_sr = g.B.s_row;
   p.C = g.C; p.tc = g.c_type; p.ldc = g.ldc;
   p.Cin = g.Cin; p.tcin = g.cin_type;
-  p.epi = g.epi; p.upper_only = g.upper_only;
+  p.epi = g.epi; p.upper_only = g.upper_only; p.row_off = g.row_off;
   const int64_t lda = g.A.s_col == 1 ? g.A.s_row : g.A.s_col;
   p.a_vec = ((uintptr_t)g.A.p % 16 == 0) && ((lda * (int64_t)dtype_size(g.A.type)) % 16 == 0);
   p.b_vec = ((uintptr_t)g.B.p % 16 == 0) && ((g.B.s_row * (int64_t)dtype_size(g.B.type)) % 16 == 0);

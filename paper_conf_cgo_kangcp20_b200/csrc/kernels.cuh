@@ -43,6 +43,7 @@ struct GemmArgs {
   int epi;
   double alpha, beta, div;   // fp64 literals (rounded to T on the device side)
   int upper_only;       // SYRK: skip tiles strictly below the diagonal
+  int64_t row_off;      // upper_only: global index of row 0 of C (row-sharded reference)
   int T;                // compute type PS_F32 / PS_F64
 };
 // R3-exact SIMT contraction (FFMA / DFMA fma chains, k ascending)

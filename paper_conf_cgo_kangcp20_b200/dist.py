@@ -2,8 +2,12 @@
 one NCCL gather of the fixed-size result records.
 
 Configurations are independent units, so the data path has no collective: every
-rank binds its own copy of the inputs, computes the fp64 reference itself and
-runs ``ps_sweep`` over its share.  The only exchange is an
+rank binds its own copy of the inputs and runs ``ps_sweep`` over its share.  The
+fp64 reference (a0) of a contraction app is sharded by contiguous output rows
+(``ps_app_reference_rows``, work-balanced for the triangular SYRK-like outputs),
+all-gathered (NCCL) and merged (``ps_app_reference_merge``) -- bit-identical to
+the single-GPU reference; the mat-vec / stencil references are one streaming
+pass and every rank computes them whole.  The only exchange is an
 ``all_gather_into_tensor`` of the 64-byte ``ps_result`` records (padded to the
 largest share), after which every rank holds the full table sorted by config id
 and picks the same best configuration (fastest passing, ties -> lowest id,
@@ -155,6 +159,62 @@ def best_index(table: np.ndarray) -> int:
     t = table["total_ms"][ok]
     cand = ok[t == t.min()]
     return int(cand[np.argmin(table["config_id"][cand])])
+
+
+# -------------------------------------------------------- sharded reference
+def row_bounds(rows: int, world: int, triangular: bool = False) -> list:
+    """Contiguous row split [b_0=0, b_1, .., b_world=rows].  Triangular outputs (row i
+    costs rows - i: upper tiles) are balanced on the cumulative cost."""
+    if not triangular:
+        return [rows * r // world for r in range(world + 1)]
+    w = np.arange(rows, 0, -1, dtype=np.float64)          # cost of row i = rows - i
+    cum = np.concatenate([[0.0], np.cumsum(w)])
+    tot = cum[-1]
+    b = [0]
+    for r in range(1, world):
+        b.append(int(np.searchsorted(cum, tot * r / world, side="left")))
+    b.append(rows)
+    for r in range(1, world + 1):                           # monotone
+        b[r] = max(b[r], b[r - 1])
+    return b
+
+
+def gather_rows(full, bounds, rank: int, cols: int, group=None):
+    """All-gather contiguous row blocks of a (rows x cols) row-major tensor in place:
+    rank r owns rows [bounds[r], bounds[r+1]).  Blocks are padded to the largest and
+    moved with one all_gather_into_tensor (NCCL over NVLink; gloo in the CPU tests)."""
+    import torch
+    import torch.distributed as dist
+    world = len(bounds) - 1
+    mx = max(bounds[r + 1] - bounds[r] for r in range(world))
+    if mx == 0:
+        return full
+    v = full.view(-1, cols)
+    send = torch.zeros(mx, cols, dtype=full.dtype, device=full.device)
+    mine = bounds[rank + 1] - bounds[rank]
+    send[:mine] = v[bounds[rank]:bounds[rank + 1]]
+    recv = torch.empty(world * mx, cols, dtype=full.dtype, device=full.device)
+    dist.all_gather_into_tensor(recv, send, group=group)
+    for r in range(world):
+        n = bounds[r + 1] - bounds[r]
+        if r != rank and n:
+            v[bounds[r]:bounds[r + 1]] = recv[r * mx:r * mx + n]
+    return full
+
+
+def sharded_reference(app, world: int, rank: int, group=None, refs=None):
+    """a0 over `world` ranks: each computes its rows of the contraction output, one
+    all-gather, then the merge (mirror) -- identical to ``app.reference()``.
+    Non-shardable apps (mat-vec, stencils) compute the whole reference locally."""
+    rows = app.shard_rows
+    if world <= 1 or rows == 0:
+        return app.reference(refs=refs)
+    refs = refs if refs is not None else app.alloc_refs()
+    bounds = row_bounds(rows, world, app.shard_triangular)
+    app.reference_rows(bounds[rank], bounds[rank + 1], refs)
+    m = next(k for k, o in enumerate(app.objects) if o["is_output"])
+    gather_rows(refs[m], bounds, rank, int(app.objects[m]["cols"]), group)
+    return app.reference_merge(refs)
 
 
 def env_rank():

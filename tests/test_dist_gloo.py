@@ -88,3 +88,63 @@ def test_gather_world2_gloo(world):
     assert len({o[2] for o in out}) == 1
     assert out[0][2] == D.best_index(expect)
     assert sum(o[3] for o in out) == 243 and min(o[3] for o in out) > 0
+
+
+# ------------------------------------------------------------ sharded reference
+@pytest.mark.parametrize("triangular", [False, True])
+def test_row_bounds_cover_and_balance(triangular):
+    for rows in (1, 7, 100, 8192):
+        for world in (1, 2, 3, 8):
+            b = D.row_bounds(rows, world, triangular)
+            assert len(b) == world + 1 and b[0] == 0 and b[-1] == rows
+            assert all(b[r] <= b[r + 1] for r in range(world))
+            cost = (lambda i: rows - i) if triangular else (lambda i: 1)
+            loads = [sum(cost(i) for i in range(b[r], b[r + 1])) for r in range(world)]
+            total = sum(loads)
+            assert max(loads) <= total / world + cost(0) + 1e-9
+
+
+def _rows_worker(rank, world, port, kind, dims, q):
+    """Each rank holds only its rows of the oracle's fp64 reference (the rest NaN, the
+    strictly-lower part of triangular outputs garbage, as ps_app_reference_rows leaves
+    them); gather_rows must reassemble every row on every rank."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_cgo_kangcp20_b200 import inputs as gen
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    objs = oracle.app_objects(kind, dims)
+    ins = gen.make_inputs(kind, objs, "random")
+    ref = oracle.reference(kind, dims, ins)
+    m = next(k for k, o in enumerate(objs) if o["is_output"])
+    rows, cols = objs[m]["rows"], objs[m]["cols"]
+    tri = kind in ("syrk", "corr", "covar")
+    b = D.row_bounds(rows, world, tri)
+    mine = np.full((rows, cols), np.nan)
+    want = ref[m].reshape(rows, cols)
+    mine[b[rank]:b[rank + 1]] = want[b[rank]:b[rank + 1]]
+    full = torch.from_numpy(mine.reshape(-1).copy())
+    D.gather_rows(full, b, rank, cols)
+    q.put((rank, full.numpy().tobytes()))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("kind,dims", [("corr", [37, 29]), ("2mm", [21, 17, 13, 11])])
+def test_gather_rows_world2_gloo(kind, dims):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rows_worker, args=(r, 2, port, kind, dims, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = sorted(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    from paper_conf_cgo_kangcp20_b200 import inputs as gen
+    objs = oracle.app_objects(kind, dims)
+    ref = oracle.reference(kind, dims, gen.make_inputs(kind, objs, "random"))
+    m = next(k for k, o in enumerate(objs) if o["is_output"])
+    for _, raw in out:
+        got = np.frombuffer(raw, dtype=np.float64)
+        assert got.tobytes() == np.ascontiguousarray(ref[m], dtype=np.float64).reshape(-1).tobytes()
