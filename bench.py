@@ -275,8 +275,28 @@ def _sample(workload):
     return kind, dims, sdims, factor, expo
 
 
+def _oracle_batch(kind, sdims, ins, ref, ids, toq, threads):
+    """Evaluate configurations with the oracle, one per host thread (ctypes releases
+    the GIL inside the C oracle, which keeps no global state)."""
+    import oracle
+    from concurrent.futures import ThreadPoolExecutor
+    m = len(oracle.app_objects(kind, sdims))
+    if threads <= 1:
+        for c in ids:
+            oracle.evaluate(kind, sdims, decode(c, m), ins, ref, toq=toq)
+        return
+    with ThreadPoolExecutor(threads) as ex:
+        list(ex.map(lambda c: oracle.evaluate(kind, sdims, decode(c, m), ins, ref, toq=toq), ids))
+
+
+def _cycle_ids(m, k, start):
+    space = 3 ** m
+    return [(start + 7 * i) % space for i in range(k)]
+
+
 def run_reference_arm(args, rank, world):
-    """The CPU oracle as it stands (single-threaded), bounded sample per step."""
+    """The CPU oracle as it stands, one configuration per host core in parallel,
+    on a bounded sample per step."""
     import oracle
     from paper_conf_cgo_kangcp20_b200 import inputs as gen
     if rank != 0:
@@ -284,21 +304,22 @@ def run_reference_arm(args, rank, world):
     kind, dims, sdims, factor, expo = _sample(args.workload)
     objs = oracle.app_objects(kind, sdims)
     ins = gen.make_inputs(kind, objs, args.input_set)
+    cores = os.cpu_count() or 1
     t0 = time.time()
     ref = oracle.reference(kind, sdims, ins)
     t_ref = time.time() - t0
     m = len(objs)
-    cycle = [(3 ** m - 1) // 2, 3 ** m - 1, 0, 1]
     for w in range(args.warmup):
-        oracle.evaluate(kind, sdims, decode(cycle[w % len(cycle)], m), ins, ref, toq=args.toq)
+        _oracle_batch(kind, sdims, ins, ref, _cycle_ids(m, cores, w * cores), args.toq, cores)
     t0 = time.time()
     for s in range(args.steps):
-        oracle.evaluate(kind, sdims, decode(cycle[s % len(cycle)], m), ins, ref, toq=args.toq)
+        _oracle_batch(kind, sdims, ins, ref, _cycle_ids(m, cores, (args.warmup + s) * cores), args.toq,
+                      cores)
     el = time.time() - t0
-    v = args.steps / el * factor
-    sample = "%s %s: 1 configuration evaluation per step (ids cycling %s) at %s, fp64 " \
-             "reference precomputed (%.1f s); throughput extrapolated to %s by (N_s/N)^%d = %.4g" % (
-                 kind, "x".join(map(str, dims)), cycle, "x".join(map(str, sdims)), t_ref,
+    v = args.steps * cores / el * factor
+    sample = "%s %s: per step %d configurations (ids 7i+c mod 3^M), one per host thread, at %s, " \
+             "fp64 reference precomputed (%.1f s); throughput extrapolated to %s by (N_s/N)^%d = %.4g" % (
+                 kind, "x".join(map(str, dims)), cores, "x".join(map(str, sdims)), t_ref,
                  "x".join(map(str, dims)), expo, factor)
     line = {"impl": "reference", "metric": "configs evaluated/s", "value": v,
             "unit": "configs/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -306,7 +327,7 @@ def run_reference_arm(args, rank, world):
             "vs_baseline": None, "dtype": "f64/f32/f16 (per configuration)", "data": "synthetic",
             "config": {"workload": args.workload, "sample": sample, "input_set": args.input_set,
                        "toq": args.toq},
-            "cpu_baseline": {"value": v, "unit": "configs/s", "cores": 1, "kind": "oracle",
+            "cpu_baseline": {"value": v, "unit": "configs/s", "cores": cores, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": v, "unit": "configs/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
@@ -315,26 +336,38 @@ def run_reference_arm(args, rank, world):
 
 
 def cpu_baseline(args):
-    """Oracle timed on the host: the fp64 reference run (config 0) + the all-f32
-    configuration of the first app, at the sample size."""
+    """Oracle timed on the host: the fp64 reference run, then one
+    configuration single-threaded and a batch of one configuration per host core in
+    parallel, at the sample size; value = the parallel rate."""
     import oracle
     from paper_conf_cgo_kangcp20_b200 import inputs as gen
     kind, dims, sdims, factor, expo = _sample(args.workload)
     objs = oracle.app_objects(kind, sdims)
     ins = gen.make_inputs(kind, objs, args.input_set)
     m = len(objs)
-    ids = [(3 ** m - 1) // 2]
+    cores = os.cpu_count() or 1
     t0 = time.time()
     ref = oracle.reference(kind, sdims, ins)
-    for cid in ids:
-        oracle.evaluate(kind, sdims, decode(cid, m), ins, ref, toq=args.toq)
-    el = time.time() - t0
-    n_eval = 1 + len(ids)
-    return {"value": n_eval / el * factor, "unit": "configs/s", "cores": 1, "kind": "oracle",
-            "sample": "%s at %s: fp64 reference run (config 0) + config %s (all-f32), single-"
-                      "threaded C oracle, %.1f s; extrapolated to %s by (N_s/N)^%d = %.4g" % (
-                          kind, "x".join(map(str, sdims)), ids, el, "x".join(map(str, dims)),
-                          expo, factor)}
+    t_ref = time.time() - t0
+    t0 = time.time()
+    _oracle_batch(kind, sdims, ins, ref, [(3 ** m - 1) // 2], args.toq, 1)
+    t_one = time.time() - t0
+    ids = _cycle_ids(m, cores, 1)
+    t0 = time.time()
+    _oracle_batch(kind, sdims, ins, ref, ids, args.toq, cores)
+    t_par = time.time() - t0
+    lscpu = ""
+    try:
+        lscpu = [l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")][0]
+    except Exception:
+        pass
+    return {"value": cores / t_par * factor, "unit": "configs/s", "cores": cores, "kind": "oracle",
+            "cpu_model": lscpu,
+            "single_thread": {"value": 1.0 / t_one * factor, "cores": 1},
+            "sample": "%s at %s: fp64 reference %.1f s; all-f32 config single-threaded %.1f s; %d configs "
+                      "(ids 7i+1 mod 3^M) one per thread in %.1f s; plain C oracle; extrapolated to %s by "
+                      "(N_s/N)^%d = %.4g" % (kind, "x".join(map(str, sdims)), t_ref, t_one, cores, t_par,
+                                             "x".join(map(str, dims)), expo, factor)}
 
 
 # ------------------------------------------------------- whole program
