@@ -19,8 +19,11 @@ namespace ps {
 namespace simt {
 
 template <class T> struct Cfg;
-template <> struct Cfg<float> { static constexpr int BM = 128, BN = 128, BK = 16, TM = 8, TN = 8; };
-template <> struct Cfg<double> { static constexpr int BM = 128, BN = 128, BK = 8, TM = 8, TN = 8; };
+// CH: consecutive columns per thread chunk (one 16-byte shared load); a thread's TN
+// columns are TN/CH chunks spaced 16*CH apart, so 8 lanes of a quarter-warp read 128
+// contiguous bytes of B (conflict-free for 8-byte T as well as 4-byte T)
+template <> struct Cfg<float> { static constexpr int BM = 128, BN = 128, BK = 16, TM = 8, TN = 8, CH = 4; };
+template <> struct Cfg<double> { static constexpr int BM = 128, BN = 128, BK = 8, TM = 8, TN = 8, CH = 2; };
 constexpr int THREADS = 256;
 
 struct Params {
@@ -87,7 +90,7 @@ __device__ __forceinline__ void load_run(const raw_t<S> *p, T (&out)[E]) {
 template <class T, class SA, class SB, bool AK>
 __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta, T div) {
   constexpr int BM = Cfg<T>::BM, BN = Cfg<T>::BN, BK = Cfg<T>::BK;
-  constexpr int TM = Cfg<T>::TM, TN = Cfg<T>::TN;
+  constexpr int TM = Cfg<T>::TM, TN = Cfg<T>::TN, CH = Cfg<T>::CH;
   constexpr int EA = BM * BK / THREADS, EB = BK * BN / THREADS;   // elements per thread per tile
   __shared__ __align__(16) T As[2][BK][BM];
   __shared__ __align__(16) T Bs[2][BK][BN];
@@ -158,7 +161,7 @@ __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta
 #pragma unroll
       for (int i = 0; i < TM; i++) a[i] = As[buf][k][(i / 4) * (BM / 2) + ty * 4 + (i % 4)];
 #pragma unroll
-      for (int j = 0; j < TN; j++) b[j] = Bs[buf][k][(j / 4) * (BN / 2) + tx * 4 + (j % 4)];
+      for (int j = 0; j < TN; j++) b[j] = Bs[buf][k][(j / CH) * (16 * CH) + tx * CH + (j % CH)];
 #pragma unroll
       for (int i = 0; i < TM; i++)
 #pragma unroll
@@ -178,7 +181,7 @@ __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta
     if (gm >= p.M) continue;
 #pragma unroll
     for (int j = 0; j < TN; j++) {
-      const int64_t gn = n0 + (j / 4) * (BN / 2) + tx * 4 + (j % 4);
+      const int64_t gn = n0 + (j / CH) * (16 * CH) + tx * CH + (j % CH);
       if (gn >= p.N) continue;
       T r = acc[i][j];
       const int64_t idx = gm * p.ldc + gn;
