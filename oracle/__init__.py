@@ -7,7 +7,9 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
 This module is argument marshalling (ctypes + numpy) around ``oracle.c``, the
 plain single-threaded C definition of SURVEY.md §8(a) a1-a5 (see the header of
 ``oracle.c`` for the paper passages each part follows).  Precision codes:
-0 = f64, 1 = f32, 2 = f16 (descending precision).
+0 = f64, 1 = f32, 2 = f16 (descending precision); 3 = bf16 for the
+Blackwell extension, whose buffers are raw uint16 bit
+patterns here (numpy has no bfloat16; ``widen`` gives their exact values).
 """
 from __future__ import annotations
 
@@ -23,8 +25,8 @@ _SRC = os.path.join(_HERE, "oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared", "-std=c11", "-Wall"]
 
-F64, F32, F16 = 0, 1, 2
-NP_DTYPE = {F64: np.float64, F32: np.float32, F16: np.float16}
+F64, F32, F16, BF16 = 0, 1, 2, 3
+NP_DTYPE = {F64: np.float64, F32: np.float32, F16: np.float16, BF16: np.uint16}
 ROWDOT_LANES = 32
 COLSUM_CHUNK = 256
 
@@ -72,6 +74,11 @@ def lib():
                                                ctypes.POINTER(ctypes.c_int)]
             L.oracle_config_encode.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_int),
                                                ctypes.POINTER(ctypes.c_uint64)]
+            L.oracle_config_decode_radix.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_uint64,
+                                                     ctypes.POINTER(ctypes.c_int)]
+            L.oracle_config_encode_radix.argtypes = [ctypes.c_int, ctypes.c_int,
+                                                     ctypes.POINTER(ctypes.c_int),
+                                                     ctypes.POINTER(ctypes.c_uint64)]
             L.oracle_app_objects.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64),
                                              ctypes.c_int, ctypes.POINTER(ObjectInfo)]
             L.oracle_run_config.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64),
@@ -109,6 +116,14 @@ def convert(a: np.ndarray, src: int, dst: int) -> np.ndarray:
     return out
 
 
+def widen(a: np.ndarray, t: int) -> np.ndarray:
+    """Exact float64 values of a buffer stored in precision t (bf16: raw uint16)."""
+    a = np.ascontiguousarray(a)
+    if t == F64:
+        return a.astype(np.float64)
+    return convert(a, t, F64)
+
+
 # ------------------------------------------------------------------- quality
 def quality(out: np.ndarray, out_type: int, ref: np.ndarray) -> dict:
     out = np.ascontiguousarray(out)
@@ -121,17 +136,17 @@ def quality(out: np.ndarray, out_type: int, ref: np.ndarray) -> dict:
 
 
 # --------------------------------------------------------------------- codec
-def config_decode(num_objects: int, cid: int) -> list:
+def config_decode(num_objects: int, cid: int, radix: int = 3) -> list:
     p = (ctypes.c_int * num_objects)()
-    if lib().oracle_config_decode(num_objects, cid, p):
+    if lib().oracle_config_decode_radix(num_objects, radix, cid, p):
         raise ValueError("bad config id")
     return list(p)
 
 
-def config_encode(prec) -> int:
+def config_encode(prec, radix: int = 3) -> int:
     p = (ctypes.c_int * len(prec))(*prec)
     out = ctypes.c_uint64()
-    if lib().oracle_config_encode(len(prec), p, ctypes.byref(out)):
+    if lib().oracle_config_encode_radix(len(prec), radix, p, ctypes.byref(out)):
         raise ValueError("bad precision vector")
     return int(out.value)
 

@@ -34,8 +34,8 @@
 /* ===================================================================== */
 
 typedef struct { int ebits, mbits, bias; } fmt_t;
-/* index = precision code: f64, f32, f16 */
-static const fmt_t FMT[3] = { {11, 52, 1023}, {8, 23, 127}, {5, 10, 15} };
+/* index = precision code: f64, f32, f16, bf16 (8 exponent, 7 fraction bits) */
+static const fmt_t FMT[4] = { {11, 52, 1023}, {8, 23, 127}, {5, 10, 15}, {8, 7, 127} };
 
 /* number of significant bits of v (0 for v == 0) */
 static int bitlen64(uint64_t v) { return v ? 64 - __builtin_clzll(v) : 0; }
@@ -111,7 +111,7 @@ static void store_bits(void *p, int t, size_t i, uint64_t b) {
 
 int oracle_convert(const void *src, int st, void *dst, int dt, size_t n) {
   size_t i;
-  if (st < 0 || st > 2 || dt < 0 || dt > 2) return 1;
+  if (st < 0 || st > 3 || dt < 0 || dt > 3) return 1;
   if (n && (!src || !dst)) return 1;
   for (i = 0; i < n; i++) {
     uint64_t b = load_bits(src, st, i);
@@ -153,7 +153,7 @@ int oracle_quality(const void *out, int ot, const double *ref, size_t n,
                    oracle_quality_result *res) {
   double s = 0.0, mx = 0.0;
   uint64_t nf = 0;
-  if (!res || ot < 0 || ot > 2) return 1;
+  if (!res || ot < 0 || ot > 3) return 1;
   oracle_quality_accumulate(out, ot, ref, n, &s, &mx, &nf);
   res->n = n;
   res->mean_rel = n ? s / (double)n : 0.0;
@@ -167,27 +167,32 @@ int oracle_quality(const void *out, int ot, const double *ref, size_t n,
 /* c-2: configuration codec                                              */
 /* ===================================================================== */
 
-int oracle_config_decode(int m, uint64_t id, int *prec) {
+/* id = sum_m code(m) * radix^m, object 0 least significant */
+int oracle_config_decode_radix(int m, int radix, uint64_t id, int *prec) {
   int i;
   uint64_t space = 1;
-  for (i = 0; i < m; i++) space *= 3;
+  if (radix != 3 && radix != 4) return 1;
+  for (i = 0; i < m; i++) space *= (uint64_t)radix;
   if (m <= 0 || id >= space || !prec) return 1;
-  for (i = 0; i < m; i++) { prec[i] = (int)(id % 3); id /= 3; }
+  for (i = 0; i < m; i++) { prec[i] = (int)(id % (uint64_t)radix); id /= (uint64_t)radix; }
   return 0;
 }
 
-int oracle_config_encode(int m, const int *prec, uint64_t *id) {
+int oracle_config_encode_radix(int m, int radix, const int *prec, uint64_t *id) {
   int i;
   uint64_t v = 0, w = 1;
-  if (m <= 0 || !prec || !id) return 1;
+  if (m <= 0 || !prec || !id || (radix != 3 && radix != 4)) return 1;
   for (i = 0; i < m; i++) {
-    if (prec[i] < 0 || prec[i] > 2) return 1;
+    if (prec[i] < 0 || prec[i] >= radix) return 1;
     v += (uint64_t)prec[i] * w;
-    w *= 3;
+    w *= (uint64_t)radix;
   }
   *id = v;
   return 0;
 }
+
+int oracle_config_decode(int m, uint64_t id, int *prec) { return oracle_config_decode_radix(m, 3, id, prec); }
+int oracle_config_encode(int m, const int *prec, uint64_t *id) { return oracle_config_encode_radix(m, 3, prec, id); }
 
 /* ===================================================================== */
 /* R1/R2/R4: objects and arithmetic "in T"                               */
@@ -218,11 +223,12 @@ static void st(obj_t *o, size_t i, double v, int T) {
   if (o->type == OR_F64) { ((double *)o->p)[i] = v; return; }
   if (T == OR_F64) b = oracle_convert_bits(double_to_bits(v), OR_F64, o->type);
   else if (o->type == OR_F32) b = float_to_bits((float)v);        /* exact: v is f32 */
-  else b = oracle_convert_bits(float_to_bits((float)v), OR_F32, OR_F16);
+  else b = oracle_convert_bits(float_to_bits((float)v), OR_F32, o->type);   /* f16 / bf16 */
   store_bits(o->p, o->type, i, b);
 }
 
-/* R2: T = widest of the touched objects, floored at f32 (code 0 = widest) */
+/* R2: T = widest of the touched objects, floored at f32 (code 0 = widest; f16 and
+ * bf16, codes 2 and 3, are both narrower than f32, so they compute in f32) */
 static int W2(int a, int b) { int t = a < b ? a : b; return t < OR_F32 ? t : OR_F32; }
 static int W3(int a, int b, int c) { return W2(W2(a, b), c); }
 
@@ -738,7 +744,7 @@ static int run_to_objects(const char *kind, const int64_t *dims, int ndims, cons
   shapes(a, d, rows, cols);
   memset(o, 0, sizeof(obj_t) * 8);
   for (m = 0; m < a->nobj; m++) {
-    if (prec[m] < 0 || prec[m] > 2) { free_objects(o, m); return 1; }
+    if (prec[m] < 0 || prec[m] > 3) { free_objects(o, m); return 1; }
     o[m].type = prec[m];
     o[m].n = (size_t)(rows[m] * cols[m]);
     o[m].p = calloc(o[m].n ? o[m].n : 1, tsize(prec[m]));
@@ -853,7 +859,7 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
   shapes(a, d, R, C);
   memset(in, 0, sizeof(in));
   for (t = 0; t < a->nobj; t++) {
-    if (prec[t] < 0 || prec[t] > 2) return 1;
+    if (prec[t] < 0 || prec[t] > 3) return 1;
     in[t].type = prec[t];
     in[t].n = (size_t)(R[t] * C[t]);
     if (a->roles[t] == 0 || a->roles[t] == 2) {

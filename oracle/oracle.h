@@ -11,7 +11,10 @@
  * readings.
  *
  * Precision codes follow the paper's descending-precision order:
- *   0 = f64, 1 = f32, 2 = f16.
+ *   0 = f64, 1 = f32, 2 = f16; and, for the Blackwell extension of SURVEY §8(f)
+ *   NEXT #4 (B200 tensor-core formats beyond the paper's fp16), 3 = bf16
+ *   (IEEE-style binary16 with 8 exponent / 7 fraction bits).  The extended
+ *   configuration space is 4^M (radix 4, same digit order).
  */
 #ifndef PRESCALER_ORACLE_H
 #define PRESCALER_ORACLE_H
@@ -22,7 +25,7 @@
 extern "C" {
 #endif
 
-enum { OR_F64 = 0, OR_F32 = 1, OR_F16 = 2 };
+enum { OR_F64 = 0, OR_F32 = 1, OR_F16 = 2, OR_BF16 = 3 };
 
 /* ---- c-1: software IEEE-754 conversion (bit manipulation only) ---------- */
 uint64_t oracle_convert_bits(uint64_t bits, int src_type, int dst_type);
@@ -47,6 +50,9 @@ int oracle_quality(const void *out, int out_type, const double *ref, size_t n,
 /* ---- c-2: configuration codec ((1+#ConvTypes)^N) ----------------- */
 int oracle_config_decode(int num_objects, uint64_t id, int *prec);
 int oracle_config_encode(int num_objects, const int *prec, uint64_t *id);
+/* radix 3 (f64, f32, f16: the paper's space) or 4 (+ bf16) */
+int oracle_config_decode_radix(int num_objects, int radix, uint64_t id, int *prec);
+int oracle_config_encode_radix(int num_objects, int radix, const int *prec, uint64_t *id);
 
 /* ---- c-4: applications ------------------------------------------------ */
 /* Reduction-order parameters (R5).  They are part of the definition. */

@@ -7,6 +7,10 @@
  *                midpoint sets + random bit patterns
  *   f64 -> f32 : SSE2 cvtsd2ss under MXCSR RNE, FTZ/DAZ off
  *   f16 -> f64, f32 -> f64 : exact C widening
+ *   f32 -> bf16: AVX512-BF16 vcvtneps2bf16 (RNE), all 2^32 inputs whose input
+ *                and result are normal or zero (the instruction flushes
+ *                subnormals: those are pinned in test_oracle_bf16.py instead)
+ *   bf16 -> f32: the definition (bits << 16), all 2^16 inputs
  * NaN inputs compare NaN-ness only (the oracle canonicalises, reading #5).
  * Usage: hwcheck <mode> [count]; prints "mismatches=<n> checked=<m>".
  */
@@ -56,6 +60,14 @@ static uint32_t hw_f64_f32(uint64_t b) {
   return o;
 }
 
+__attribute__((target("avx512bf16,avx512vl"))) static uint16_t hw_f32_bf16(uint32_t b) {
+  float f;
+  memcpy(&f, &b, 4);
+  __m128bh r = _mm_cvtneps_pbh(_mm_set_ss(f));
+  return (uint16_t)_mm_extract_epi16((__m128i)r, 0);
+}
+static int is_nan_bf16(uint64_t h) { return ((h >> 7) & 0xFF) == 0xFF && (h & 0x7F); }
+
 static uint64_t check_f64_f16(uint64_t b, int *has_nan_ok) {
   uint64_t o = oracle_convert_bits(b, OR_F64, OR_F16), h = hw_f64_f16(b);
   *has_nan_ok = is_nan64(b) && is_nan16(o) && is_nan16(h);
@@ -76,6 +88,34 @@ int main(int argc, char **argv) {
         if (o != h && !(is_nan32(b) && is_nan16(o) && is_nan16(h))) bad++;
         checked++;
       }
+    }
+  } else if (!strcmp(mode, "f32bf16")) {         /* all 2^32 inputs (normal/zero) */
+    if (!__builtin_cpu_supports("avx512bf16")) { printf("skip=noavx512bf16\n"); return 0; }
+#pragma omp parallel for reduction(+ : bad, checked) schedule(static)
+    for (int64_t hi = 0; hi < 65536; hi++) {
+      for (uint32_t lo = 0; lo < 65536; lo++) {
+        uint32_t b = ((uint32_t)hi << 16) | lo;
+        uint64_t o = oracle_convert_bits(b, OR_F32, OR_BF16), h;
+        if (((b >> 23) & 0xFF) == 0 && (b & 0x7FFFFF)) continue;     /* subnormal input */
+        if (((o >> 7) & 0xFF) == 0 && (o & 0x7F)) continue;           /* subnormal result */
+        h = hw_f32_bf16(b);
+        if (o != h && !(is_nan32(b) && is_nan_bf16(o) && is_nan_bf16(h))) bad++;
+        checked++;
+      }
+    }
+  } else if (!strcmp(mode, "bf16wide")) {        /* all 2^16 inputs: exact widening */
+    for (uint32_t h = 0; h < 65536; h++) {
+      uint64_t o32 = oracle_convert_bits(h, OR_BF16, OR_F32), o64 = oracle_convert_bits(h, OR_BF16, OR_F64);
+      uint32_t w = h << 16;
+      float f;
+      double d;
+      uint64_t w64;
+      memcpy(&f, &w, 4);
+      d = (double)f;
+      memcpy(&w64, &d, 8);
+      if (is_nan_bf16(h)) bad += !(is_nan32(o32) && is_nan64(o64));
+      else bad += (o32 != w) + (o64 != w64);
+      checked++;
     }
   } else if (!strcmp(mode, "f16wide")) {         /* all 2^16 inputs, both widenings */
     if (!__builtin_cpu_supports("f16c")) { printf("skip=nof16c\n"); return 0; }
