@@ -35,8 +35,11 @@
 extern "C" {
 #endif
 
-/* precision codes in the paper's descending-precision order */
-typedef enum { PS_F64 = 0, PS_F32 = 1, PS_F16 = 2 } ps_dtype;
+/* precision codes in the paper's descending-precision order; PS_BF16
+ * is the Blackwell extension (reading #28): raw
+ * uint16 bit patterns (1 sign, 8 exponent, 7 fraction bits), RNE narrowing with
+ * subnormals, overflow to inf, canonical NaN 0x7FFF. */
+typedef enum { PS_F64 = 0, PS_F32 = 1, PS_F16 = 2, PS_BF16 = 3 } ps_dtype;
 
 typedef enum {
   PS_OK = 0,
@@ -113,7 +116,11 @@ PS_API int ps_app_num_objects(const ps_app *app);            /* -1 if app == NUL
 PS_API ps_status ps_app_object_info(const ps_app *app, int m, ps_object_info *out);
 /* flags: PS_FLAG_NO_TENSOR_CORES forces the SIMT contraction path for fp16   */
 /* operands (bit-exact with R3) instead of tcgen05 (tolerance R6).            */
+/* PS_FLAG_BF16 extends the configuration alphabet to {f64, f32, f16, bf16}:  */
+/* precision vectors may hold PS_BF16 and ids run over 4^M (radix 4, object 0 */
+/* least significant); without it the space is the paper's 3^M.               */
 #define PS_FLAG_NO_TENSOR_CORES 1u
+#define PS_FLAG_BF16 2u
 PS_API ps_status ps_app_set_flags(ps_app *app, uint32_t flags);
 /* Device workspace the caller must allocate (>= 256-byte aligned). */
 PS_API size_t ps_app_workspace_bytes(const ps_app *app);

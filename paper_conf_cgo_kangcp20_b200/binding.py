@@ -17,8 +17,10 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libprescaler.so")
 
 F64, F32, F16 = 0, 1, 2                      # ps_dtype (descending precision)
+BF16 = 3                                     # Blackwell extension (reading #28)
 METRIC_MRE, METRIC_MAX_REL = 0, 1
 FLAG_NO_TENSOR_CORES = 1
+FLAG_BF16 = 2                                # configuration alphabet {f64, f32, f16, bf16}: 4^M
 ROLE_IN, ROLE_OUT, ROLE_INOUT, ROLE_TEMP = 0, 1, 2, 3
 
 # every symbol include/prescaler.h declares
@@ -241,6 +243,7 @@ class App:
                                      cols=info.cols, orig=info.orig, role=info.role,
                                      is_output=bool(info.is_output)))
         self.workspace_bytes = int(lib().ps_app_workspace_bytes(h))
+        self.flags = 0
         self._keep = []
         self.inputs = self.outputs = self.ref = None
 
@@ -256,11 +259,16 @@ class App:
             pass
 
     @property
+    def radix(self) -> int:
+        return 4 if self.flags & FLAG_BF16 else 3
+
+    @property
     def space(self) -> int:
-        return 3 ** self.num_objects
+        return self.radix ** self.num_objects
 
     def set_flags(self, flags: int):
         _check(lib().ps_app_set_flags(self._h, flags), "ps_app_set_flags")
+        self.flags = int(flags)
 
     def bind(self, inputs, outputs=None, workspace=None, device=None):
         """inputs: per object an f32 CUDA tensor (role in/inout) or None.

@@ -295,8 +295,10 @@ inline void *eoff(const void *p, int type, int64_t n) {
 }
 
 ps_status contraction(Ctx &c, GemmArgs g) {
-  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && g.A.type == PS_F16 &&
-                  g.B.type == PS_F16 && g.T == PS_F32 && g.row_off == 0 && gemm_tc_supported(g);
+  // tcgen05 for fp16 x fp16 or bf16 x bf16 multiplicands (kind::f16), f32 compute
+  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && g.A.type == g.B.type &&
+                  (g.A.type == PS_F16 || g.A.type == PS_BF16) && g.T == PS_F32 && g.row_off == 0 &&
+                  gemm_tc_supported(g);
   return tc ? gemm_tc_async(g, c.st) : gemm_simt_async(g, c.st);
 }
 
@@ -441,10 +443,16 @@ ps_status run_statements(Ctx &c) {
   return PS_OK;
 }
 
+// configuration alphabet: the paper's {f64, f32, f16}, or + bf16 (PS_FLAG_BF16, reading #28)
+int radix(const ps_app *a) { return (a->flags & PS_FLAG_BF16) ? 4 : 3; }
+
 ps_status check_prec(const ps_app *a, const int *prec) {
   if (!prec) { set_error("null precision vector"); return PS_ERR_INVALID; }
   for (int m = 0; m < a->def->nobj; m++)
-    if (!dtype_ok(prec[m])) { set_error("bad precision code %d for object %d", prec[m], m); return PS_ERR_INVALID; }
+    if (!dtype_ok(prec[m]) || prec[m] >= radix(a)) {
+      set_error("bad precision code %d for object %d (alphabet of %d)", prec[m], m, radix(a));
+      return PS_ERR_INVALID;
+    }
   return PS_OK;
 }
 
@@ -513,12 +521,13 @@ ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res
 
 uint64_t space(const ps_app *a) {
   uint64_t s = 1;
-  for (int m = 0; m < a->def->nobj; m++) s *= 3;
+  for (int m = 0; m < a->def->nobj; m++) s *= (uint64_t)radix(a);
   return s;
 }
 
 void decode(const ps_app *a, uint64_t id, int *prec) {
-  for (int m = 0; m < a->def->nobj; m++) { prec[m] = (int)(id % 3); id /= 3; }
+  const uint64_t r = (uint64_t)radix(a);
+  for (int m = 0; m < a->def->nobj; m++) { prec[m] = (int)(id % r); id /= r; }
 }
 
 uint64_t n_outputs(const ps_app *a) {
@@ -759,14 +768,17 @@ ps_status ps_config_encode(const ps_app *a, const int *prec, uint64_t *id) {
   ps_status s = check_prec(a, prec);
   if (s != PS_OK) return s;
   uint64_t v = 0, w = 1;
-  for (int m = 0; m < a->def->nobj; m++) { v += (uint64_t)prec[m] * w; w *= 3; }
+  for (int m = 0; m < a->def->nobj; m++) { v += (uint64_t)prec[m] * w; w *= (uint64_t)radix(a); }
   *id = v;
   return PS_OK;
 }
 
 ps_status ps_config_decode(const ps_app *a, uint64_t id, int *prec) {
   if (!a || !prec) { set_error("ps_config_decode: null pointer"); return PS_ERR_INVALID; }
-  if (id >= space(a)) { set_error("ps_config_decode: id %llu >= 3^%d", (unsigned long long)id, a->def->nobj); return PS_ERR_INVALID; }
+  if (id >= space(a)) {
+    set_error("ps_config_decode: id %llu >= %d^%d", (unsigned long long)id, radix(a), a->def->nobj);
+    return PS_ERR_INVALID;
+  }
   decode(a, id, prec);
   return PS_OK;
 }
@@ -979,7 +991,7 @@ ps_status ps_search(ps_app *a, double toq, int repeats, void *stream, ps_search_
   Trial tcur{0.f, 0.0, false};
   bool have = false;
   uint64_t cur_id = 0;
-  for (int t = PS_F64; t <= PS_F16; t++) {
+  for (int t = PS_F64; t < radix(a); t++) {
     for (int m = 0; m < M; m++) cand[m] = t;
     Trial tr;
     if ((s = run(cand, &tr)) != PS_OK) return s;
@@ -1014,7 +1026,7 @@ ps_status ps_search(ps_app *a, double toq, int repeats, void *stream, ps_search_
     memcpy(best, cur, sizeof(cur));
     Trial tbest = tcur;
     uint64_t best_id = cur_id;
-    for (int t = PS_F64; t <= PS_F16; t++) {          // descending precision
+    for (int t = PS_F64; t < radix(a); t++) {         // descending precision
       if (t == cur[m]) continue;                       // line 3
       memcpy(cand, cur, sizeof(cur));
       cand[m] = t;

@@ -1,6 +1,6 @@
 // common.cuh -- shared device/host helpers of libprescaler (sm_100a).
 //
-// Storage types: f64 = double, f32 = float, f16 = uint16_t bit patterns.
+// Storage types: f64 = double, f32 = float, f16 / bf16 = uint16_t bit patterns.
 // Compute type T is float or double (reading R2: widest touched precision,
 // floored at f32).  The library is compiled with -fmad=false and without
 // fast-math, so every +,-,*,/,sqrt below is one correctly rounded IEEE op in T
@@ -35,7 +35,7 @@ void count_launch();
   } while (0)
 
 inline size_t dtype_size(int t) { return t == PS_F64 ? 8 : (t == PS_F32 ? 4 : 2); }
-inline bool dtype_ok(int t) { return t == PS_F64 || t == PS_F32 || t == PS_F16; }
+inline bool dtype_ok(int t) { return t == PS_F64 || t == PS_F32 || t == PS_F16 || t == PS_BF16; }
 // R2: compute type = widest (smallest code) floored at f32
 inline int widest(int a, int b) { return a < b ? a : b; }
 inline int compute_type(std::initializer_list<int> ts) {
@@ -46,12 +46,14 @@ inline int compute_type(std::initializer_list<int> ts) {
 int num_sms();
 
 // ------------------------------------------------------- storage traits
-struct F16 { uint16_t b; };   // tag type for fp16 storage (IEEE binary16 bits)
+struct F16 { uint16_t b; };    // tag type for fp16 storage (IEEE binary16 bits)
+struct BF16 { uint16_t b; };   // tag type for bf16 storage (reading #28)
 
 template <class S> struct Store;
 template <> struct Store<double> { using raw = double; static constexpr int code = PS_F64; };
 template <> struct Store<float> { using raw = float; static constexpr int code = PS_F32; };
 template <> struct Store<F16> { using raw = uint16_t; static constexpr int code = PS_F16; };
+template <> struct Store<BF16> { using raw = uint16_t; static constexpr int code = PS_BF16; };
 
 // exact widening of a stored element to T (NaN payloads are irrelevant for
 // arithmetic: any NaN propagates and is scored as non-finite)
@@ -65,6 +67,10 @@ __device__ __forceinline__ double f16_to_f64(uint16_t h) {
   asm("cvt.f64.f16 %0, %1;" : "=d"(d) : "h"(h));
   return d;
 }
+
+// bf16 -> f32 is exact: the bf16 bits are the high half of the f32 bits
+__device__ __forceinline__ float bf16_to_f32(uint16_t h) { return __uint_as_float((uint32_t)h << 16); }
+template <class T> __device__ __forceinline__ T widen_b(uint16_t h) { return (T)bf16_to_f32(h); }
 
 template <class T> __device__ __forceinline__ T widen(float v) { return (T)v; }
 template <class T> __device__ __forceinline__ T widen(double v) { return (T)v; }
@@ -82,6 +88,9 @@ template <class T> struct Ld<float, T> {
 template <class T> struct Ld<F16, T> {
   static __device__ __forceinline__ T get(const uint16_t *p, size_t i) { return widen_h<T>(p[i]); }
 };
+template <class T> struct Ld<BF16, T> {
+  static __device__ __forceinline__ T get(const uint16_t *p, size_t i) { return widen_b<T>(p[i]); }
+};
 
 // ------------------------------------------- RNE narrowing (reading R1, c-1)
 // canonical NaN (reading #5): every bit set except the sign
@@ -94,6 +103,17 @@ __device__ __forceinline__ uint16_t rne_f16(float x) {
 __device__ __forceinline__ uint16_t rne_f16(double x) {
   uint16_t h;
   asm("cvt.rn.f16.f64 %0, %1;" : "=h"(h) : "d"(x));
+  return (x != x) ? (uint16_t)0x7FFF : h;
+}
+// bf16 (reading #28): one RNE rounding from f32 or from f64 (F2F.BF16.F64)
+__device__ __forceinline__ uint16_t rne_bf16(float x) {
+  uint16_t h;
+  asm("cvt.rn.bf16.f32 %0, %1;" : "=h"(h) : "f"(x));
+  return (x != x) ? (uint16_t)0x7FFF : h;
+}
+__device__ __forceinline__ uint16_t rne_bf16(double x) {
+  uint16_t h;
+  asm("cvt.rn.bf16.f64 %0, %1;" : "=h"(h) : "d"(x));
   return (x != x) ? (uint16_t)0x7FFF : h;
 }
 __device__ __forceinline__ float rne_f32(double x) {
@@ -122,6 +142,9 @@ template <> struct St<float, double> {
 template <class T> struct St<F16, T> {
   static __device__ __forceinline__ void put(uint16_t *p, size_t i, T v) { p[i] = rne_f16(v); }
 };
+template <class T> struct St<BF16, T> {
+  static __device__ __forceinline__ void put(uint16_t *p, size_t i, T v) { p[i] = rne_bf16(v); }
+};
 
 // R4 arithmetic helpers (explicit FMA; everything else is plain IEEE)
 __device__ __forceinline__ float t_fma(float a, float b, float c) { return __fmaf_rn(a, b, c); }
@@ -133,6 +156,7 @@ template <class F> inline ps_status dispatch_store(int t, F &&f) {
     case PS_F64: return f(double());
     case PS_F32: return f(float());
     case PS_F16: return f(F16());
+    case PS_BF16: return f(BF16());
   }
   return PS_ERR_INVALID;
 }

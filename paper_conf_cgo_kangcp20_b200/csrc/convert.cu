@@ -37,6 +37,25 @@ template <> struct Cvt<F16, double> {
 template <> struct Cvt<float, double> {
   static __device__ __forceinline__ double f(float x) { return canon_f64((double)x); }
 };
+// bf16 (reading #28): one RNE rounding from any wider format; widening is exact
+template <> struct Cvt<float, BF16> {
+  static __device__ __forceinline__ uint16_t f(float x) { return rne_bf16(x); }
+};
+template <> struct Cvt<double, BF16> {
+  static __device__ __forceinline__ uint16_t f(double x) { return rne_bf16(x); }
+};
+template <> struct Cvt<F16, BF16> {   // f16 -> f32 is exact, so one rounding
+  static __device__ __forceinline__ uint16_t f(uint16_t h) { return rne_bf16(f16_to_f32(h)); }
+};
+template <> struct Cvt<BF16, float> {
+  static __device__ __forceinline__ float f(uint16_t h) { return canon_f32(bf16_to_f32(h)); }
+};
+template <> struct Cvt<BF16, double> {
+  static __device__ __forceinline__ double f(uint16_t h) { return canon_f64((double)bf16_to_f32(h)); }
+};
+template <> struct Cvt<BF16, F16> {   // bf16 -> f32 is exact, so one rounding
+  static __device__ __forceinline__ uint16_t f(uint16_t h) { return rne_f16(bf16_to_f32(h)); }
+};
 
 // ------------------------------------------------------- vector helpers
 template <int B> struct Vec;
@@ -155,6 +174,12 @@ ps_status convert_async(const void *src, int st, void *dst, int dt, size_t n, cu
   if (st == PS_F16 && dt == PS_F32) return launch_convert<F16, float>(src, dst, n, stream);
   if (st == PS_F16 && dt == PS_F64) return launch_convert<F16, double>(src, dst, n, stream);
   if (st == PS_F32 && dt == PS_F64) return launch_convert<float, double>(src, dst, n, stream);
+  if (st == PS_F32 && dt == PS_BF16) return launch_convert<float, BF16>(src, dst, n, stream);
+  if (st == PS_F64 && dt == PS_BF16) return launch_convert<double, BF16>(src, dst, n, stream);
+  if (st == PS_F16 && dt == PS_BF16) return launch_convert<F16, BF16>(src, dst, n, stream);
+  if (st == PS_BF16 && dt == PS_F32) return launch_convert<BF16, float>(src, dst, n, stream);
+  if (st == PS_BF16 && dt == PS_F64) return launch_convert<BF16, double>(src, dst, n, stream);
+  if (st == PS_BF16 && dt == PS_F16) return launch_convert<BF16, F16>(src, dst, n, stream);
   set_error("ps_convert: bad dtype pair %d->%d", st, dt);
   return PS_ERR_INVALID;
 }

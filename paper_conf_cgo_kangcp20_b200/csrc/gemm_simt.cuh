@@ -48,6 +48,7 @@ __device__ __forceinline__ T load_elem(const void *p, int type, int64_t idx) {
   switch (type) {
     case PS_F64: return (T)((const double *)p)[idx];
     case PS_F32: return (T)((const float *)p)[idx];
+    case PS_BF16: return widen_b<T>(((const uint16_t *)p)[idx]);
     default: return widen_h<T>(((const uint16_t *)p)[idx]);
   }
 }
@@ -56,6 +57,7 @@ __device__ __forceinline__ void store_elem(void *p, int type, int64_t idx, T v) 
   switch (type) {
     case PS_F64: ((double *)p)[idx] = (double)v; break;
     case PS_F32: St<float, T>::put((float *)p, idx, v); break;
+    case PS_BF16: St<BF16, T>::put((uint16_t *)p, idx, v); break;
     default: St<F16, T>::put((uint16_t *)p, idx, v); break;
   }
 }

@@ -1,5 +1,5 @@
 // gemm_simt_f32.cu -- instantiations of the R3-exact SIMT contraction with
-// compute type f32 (operands stored in f32 or f16; FFMA chains).
+// compute type f32 (operands stored in f32, f16 or bf16; FFMA chains).
 #include "gemm_simt.cuh"
 
 namespace ps {
@@ -11,9 +11,11 @@ ps_status gemm_simt_f32(const GemmArgs &g, cudaStream_t st) {
   auto pick = [&](auto sa) -> ps_status {
     using SA = decltype(sa);
     if (g.B.type == PS_F16) return launch<float, SA, F16>(p, ak, g.alpha, g.beta, g.div, st);
+    if (g.B.type == PS_BF16) return launch<float, SA, BF16>(p, ak, g.alpha, g.beta, g.div, st);
     return launch<float, SA, float>(p, ak, g.alpha, g.beta, g.div, st);
   };
   if (g.A.type == PS_F16) return pick(F16());
+  if (g.A.type == PS_BF16) return pick(BF16());
   return pick(float());
 }
 

@@ -46,6 +46,7 @@ struct Params {
   int epi;
   float alpha, beta, div;
   int upper_only;
+  uint32_t ab_fmt;   // kind::f16 operand format: 0 = f16, 1 = bf16 (reading #28)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -123,10 +124,13 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
 }
 
 __device__ __forceinline__ float load_c(const void *p, int type, int64_t idx) {
-  return type == PS_F32 ? ((const float *)p)[idx] : f16_to_f32(((const uint16_t *)p)[idx]);
+  if (type == PS_F32) return ((const float *)p)[idx];
+  const uint16_t h = ((const uint16_t *)p)[idx];
+  return type == PS_BF16 ? bf16_to_f32(h) : f16_to_f32(h);
 }
 __device__ __forceinline__ void store_c(void *p, int type, int64_t idx, float v) {
   if (type == PS_F32) ((float *)p)[idx] = v;
+  else if (type == PS_BF16) ((uint16_t *)p)[idx] = rne_bf16(v);
   else ((uint16_t *)p)[idx] = rne_f16(v);
 }
 
@@ -191,6 +195,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   } else if (warp == 1) {
     if (lane == 0) {   // ---------------- MMA issuer (single thread)
       const uint32_t idesc = (1u << 4)                          // D = f32
+                             | (p.ab_fmt << 7) | (p.ab_fmt << 10)   // A, B format
                              | ((uint32_t)p.a_mn_major << 15)   // A major
                              | (1u << 16)                       // B is N-major
                              | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
@@ -401,7 +406,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
     }
   } else if (warp == 1) {
     if (leader && lane == 0) {   // ---- MMA issuer (leader CTA, single thread)
-      const uint32_t idesc = (1u << 4) | ((uint32_t)p.a_mn_major << 15) | (1u << 16) |
+      const uint32_t idesc = (1u << 4) | (p.ab_fmt << 7) | (p.ab_fmt << 10) |
+                             ((uint32_t)p.a_mn_major << 15) | (1u << 16) |
                              ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
       int64_t cursor = cluster;
       int m0, n0;
@@ -489,20 +495,23 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 // 2-D fp16 tensor map: inner (contiguous) extent, outer extent, outer stride in bytes,
 // box {64, box_outer}, 128-byte swizzle, zero fill out of bounds.
 static bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer,
-                     uint64_t stride_bytes, uint32_t box_outer) {
+                     uint64_t stride_bytes, uint32_t box_outer, bool bf16) {
   auto fn = encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {inner, outer};
   cuuint64_t strides[1] = {stride_bytes};
   cuuint32_t box[2] = {64, box_outer};
   cuuint32_t es[2] = {1, 1};
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
+  return fn(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 bool gemm_tc_supported(const GemmArgs &g) {
-  if (g.A.type != PS_F16 || g.B.type != PS_F16 || g.T != PS_F32) return false;
+  // both multiplicands fp16, or both bf16 (kind::f16 takes either, not a mix)
+  if (!((g.A.type == PS_F16 && g.B.type == PS_F16) || (g.A.type == PS_BF16 && g.B.type == PS_BF16)) ||
+      g.T != PS_F32)
+    return false;
   if (g.c_type == PS_F64 || (g.epi == EPI_AXPBY && g.cin_type == PS_F64)) return false;
   if (g.M <= 0 || g.N <= 0 || g.K <= 0 || g.M > (1 << 30) || g.N > (1 << 30) || g.K > (1 << 30))
     return false;
@@ -524,15 +533,16 @@ ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
   CUtensorMap ma, mb;
   const bool a_mn = !(g.A.s_col == 1);
   bool ok;
-  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * 2, BM);
-  else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * 2, 64);
-  ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * 2, 64);
+  const bool bf = g.A.type == PS_BF16;
+  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * 2, BM, bf);
+  else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * 2, 64, bf);
+  ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * 2, 64, bf);
   if (!ok) {
     set_error("cuTensorMapEncodeTiled failed");
     return PS_ERR_CUDA;
   }
   Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
-           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only};
+           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, bf ? 1u : 0u};
   if ((g.M > BM || g.N > BN) && !getenv("PS_TC_1SM")) {   // 2-CTA persistent path
     using namespace tc2;
     static bool attr2 = false;

@@ -87,6 +87,17 @@ static bool simd_ok() {
   return ok == 1;
 }
 
+// f32 -> bf16 (reading #28): RNE on the bit pattern -- the bf16 result is the high
+// half of (bits + 0x7FFF + lsb) for every finite input (subnormals included; the
+// carry into the exponent is the correct rounding up and reaches 0x7F80 = inf
+// exactly on overflow); NaN -> canonical 0x7FFF
+static inline uint16_t f32_to_bf16_scalar(float f) {
+  uint32_t b;
+  memcpy(&b, &f, 4);
+  if ((b & 0x7F800000u) == 0x7F800000u && (b & 0x7FFFFFu)) return (uint16_t)0x7FFF;
+  return (uint16_t)((b + 0x7FFFu + ((b >> 16) & 1u)) >> 16);
+}
+
 // One contiguous range, SIMD when available (Fig. 3b) or a plain scalar loop (Fig. 3a).
 static void convert_range(const float *s, void *d, int dt, size_t n, bool simd) {
   if (dt == PS_F32) {
@@ -95,6 +106,9 @@ static void convert_range(const float *s, void *d, int dt, size_t n, bool simd) 
     uint16_t *o = (uint16_t *)d;
     if (simd && simd_ok()) f16_simd(s, o, n);
     else for (size_t i = 0; i < n; i++) o[i] = f32_to_f16_scalar(s[i]);
+  } else if (dt == PS_BF16) {   // integer-only rounding: the compiler vectorises the loop
+    uint16_t *o = (uint16_t *)d;
+    for (size_t i = 0; i < n; i++) o[i] = f32_to_bf16_scalar(s[i]);
   } else {
     double *o = (double *)d;
     if (simd && simd_ok()) f64_simd(s, o, n);

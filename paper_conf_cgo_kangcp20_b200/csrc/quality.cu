@@ -42,6 +42,10 @@ template <> struct Deliver<F16> {
   static __device__ __forceinline__ float f(uint16_t h) { return canon_f32(f16_to_f32(h)); }
   static __device__ __forceinline__ double exact(uint16_t h) { return f16_to_f64(h); }
 };
+template <> struct Deliver<BF16> {
+  static __device__ __forceinline__ float f(uint16_t h) { return canon_f32(bf16_to_f32(h)); }
+  static __device__ __forceinline__ double exact(uint16_t h) { return (double)bf16_to_f32(h); }
+};
 
 __device__ __forceinline__ void block_reduce3(double &sum, double &mx, unsigned long long &nf,
                                               double *s_sum, double *s_mx,

@@ -13,6 +13,7 @@ template <class A> struct Wider<A, double> { using t = double; };
 template <> struct Wider<double, double> { using t = double; };
 template <class S> struct CT { using t = typename Wider<S, float>::t; };   // storage -> min compute
 template <> struct CT<F16> { using t = float; };
+template <> struct CT<BF16> { using t = float; };
 // R2: T = W(objects touched, f32)
 template <class A, class B, class C>
 using T3 = typename Wider<typename Wider<typename CT<A>::t, typename CT<B>::t>::t,
@@ -31,6 +32,7 @@ __device__ __forceinline__ T load_any(const void *p, int type, int64_t i) {
   switch (type) {
     case PS_F64: return (T)__ldg((const double *)p + i);
     case PS_F32: return (T)__ldg((const float *)p + i);
+    case PS_BF16: return widen_b<T>(__ldg((const unsigned short *)p + i));
     default: return widen_h<T>(__ldg((const unsigned short *)p + i));
   }
 }

@@ -201,4 +201,4 @@ def decide(app, host_inputs, db: dict, toq: float = 0.9, threads: int = 0, verif
 
     return {"prec": list(cur), "methods": list(cur_m), "method_names": [NAMES[m] for m in cur_m],
             "result": cur_r, "pfp": pfp, "trials": len(log), "log": log,
-            "space": 3 ** M}
+            "space": app.space}

@@ -26,8 +26,8 @@ import os
 
 import numpy as np
 
-F64, F32, F16 = 0, 1, 2
-SIZE = {F64: 8, F32: 4, F16: 2}
+F64, F32, F16, BF16 = 0, 1, 2, 3
+SIZE = {F64: 8, F32: 4, F16: 2, BF16: 2}
 # nominal B200 rates for the cost model (only relative values matter)
 HBM_BPS = 6.5e12
 PEAK = {"tc": 1.2e15, F32: 60e12, F64: 30e12}
@@ -68,18 +68,18 @@ def _statements(kind, d):
     raise KeyError(kind)
 
 
-def decode(cid: int, m: int) -> list:
+def decode(cid: int, m: int, radix: int = 3) -> list:
     out = []
     for _ in range(m):
-        out.append(cid % 3)
-        cid //= 3
+        out.append(cid % radix)
+        cid //= radix
     return out
 
 
-def config_cost(kind: str, dims, objects, cid: int) -> float:
+def config_cost(kind: str, dims, objects, cid: int, radix: int = 3) -> float:
     """Predicted seconds for one configuration (deterministic, identical on all ranks)."""
     m = len(objects)
-    p = decode(cid, m)
+    p = decode(cid, m, radix)
     d = list(dims) if len(dims) > 1 else list(dims) * 5
     n = [int(o["rows"]) * int(o["cols"]) for o in objects]
     t = 0.0
@@ -96,7 +96,8 @@ def config_cost(kind: str, dims, objects, cid: int) -> float:
         else:
             _, a, b, out, (M, N, K) = st
             T = F64 if F64 in (p[a], p[b], p[out]) else F32
-            peak = PEAK["tc"] if (p[a] == F16 and p[b] == F16 and T == F32) else PEAK[T]
+            tc = p[a] == p[b] and p[a] in (F16, BF16) and T == F32
+            peak = PEAK["tc"] if tc else PEAK[T]
             t += 2.0 * M * N * K / peak
     return t
 
@@ -114,8 +115,8 @@ def lpt_partition(costs, world: int) -> list:
     return [sorted(p) for p in parts]
 
 
-def partition_configs(kind, dims, objects, config_ids, world: int, rank: int) -> list:
-    costs = [config_cost(kind, dims, objects, c) for c in config_ids]
+def partition_configs(kind, dims, objects, config_ids, world: int, rank: int, radix: int = 3) -> list:
+    costs = [config_cost(kind, dims, objects, c, radix) for c in config_ids]
     parts = lpt_partition(costs, world)
     return [config_ids[i] for i in parts[rank]]
 
