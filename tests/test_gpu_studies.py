@@ -63,3 +63,14 @@ def test_fig12_choice_passes_toq(torch):
             assert 0.0 <= r["half_fraction"] <= 1.0 and r["trials"] <= 3 * len(objs) + 3 + 2 * len(objs)
             dev = r["device_only_exhaustive"]
             assert dev is not None and dev["passing"] >= 1
+
+
+def test_bf16_gain_structure(torch):
+    from paper_conf_cgo_kangcp20_b200 import studies
+    res = studies.bf16_gain(torch, {"gemm": [64], "atax": [300, 70]}, input_sets=("default",))
+    for kind, row in res.items():
+        r = row["default"]
+        # the 4^M space contains the 3^M one: at least as many passing configs, and a
+        # best that is no slower than the paper-space best (up to timing noise)
+        assert r["bf16_4^M"]["passing"] >= r["paper_3^M"]["passing"]
+        assert r["bf16_4^M"]["space"] == 4 ** len(r["bf16_4^M"]["best_prec"])
