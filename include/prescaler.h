@@ -17,7 +17,8 @@
  *  - Every call returns ps_status.  No C++ exception crosses the ABI.  Errors of
  *    asynchronous work surface at the next synchronising call as PS_ERR_CUDA.
  *    ps_last_error() returns a thread-local message for the last failure.
- *  - Buffers of a dtype hold IEEE binary64 / binary32 / binary16 values.
+ *  - Buffers of a dtype hold IEEE binary64 / binary32 / binary16 values, or
+ *    bfloat16 bit patterns (PS_BF16).
  *  - One ps_app per host thread / stream (not thread-safe per handle).
  */
 #ifndef PRESCALER_H
@@ -43,7 +44,7 @@ typedef enum { PS_F64 = 0, PS_F32 = 1, PS_F16 = 2, PS_BF16 = 3 } ps_dtype;
 
 typedef enum {
   PS_OK = 0,
-  PS_ERR_INVALID = 1,      /* null pointer, bad dtype, id >= 3^M, wrong ndims, overlap */
+  PS_ERR_INVALID = 1,      /* null pointer, bad dtype, id >= radix^M, wrong ndims      */
   PS_ERR_UNSUPPORTED = 2,  /* unknown app kind / dims out of range                    */
   PS_ERR_CUDA = 3,         /* CUDA runtime error (message in ps_last_error())          */
   PS_ERR_WORKSPACE = 4     /* workspace missing or smaller than ps_app_workspace_bytes */
@@ -64,8 +65,9 @@ PS_API uint64_t ps_kernel_launches(void);
 /* ------------------------------------------------------------------------- */
 /* (1) Device-side type conversion of one memory object (Fig. 3c). */
 /*   dst[i] = RNE_{dst_type}(src[i]) for i < n; widening is exact; subnormals   */
-/*   kept; overflow -> +-inf; NaN -> canonical NaN (f16 0x7FFF, f32 0x7FFFFFFF, */
-/*   f64 0x7FFFFFFFFFFFFFFF).  f64 -> f16 is a single rounding.  src, dst: device */
+/*   kept; overflow -> +-inf; NaN -> canonical NaN (f16 / bf16 0x7FFF, f32      */
+/*   0x7FFFFFFF, f64 0x7FFFFFFFFFFFFFFF).  f64 -> f16 and f64 -> bf16 are single */
+/*   roundings; every pair of the four types is supported.  src, dst: device    */
 /*   pointers, any alignment (16-byte aligned pointers take the vector path);    */
 /*   overlapping ranges -> PS_ERR_INVALID; n == 0 is a no-op; src_type ==        */
 /*   dst_type is a device-to-device copy.  Asynchronous on `stream`.             */
@@ -95,6 +97,10 @@ PS_API ps_status ps_quality(const void *out, int out_type, const double *ref, si
 /*          "atax" dims {NX,NY}   "bicg" dims {NX,NY}                          */
 /*          "gesummv" dims {N}    scalars {alpha,beta} (default 43532,12313)    */
 /*          "corr" dims {N,M} scalars {eps} (default 0.005)  "covar" dims {N,M} */
+/*          "mvt" dims {N}     "syrk" dims {N,M} scalars {alpha,beta}           */
+/*          "conv2d" dims {NI,NJ}   "syr2k" dims {N,M} scalars {alpha,beta}     */
+/*          "conv3d" dims {NI,NJ,NK}   "fdtd2d" dims {TMAX,NX,NY}              */
+/*          (SYRK/SYR2K defaults 32412, 2123; readings #23-#27)                  */
 /*   ndims == 1 sets every dimension to dims[0].  scalars may be NULL.          */
 /*   Every object's original precision is f32 (BASELINE).  Object order is the  */
 /*   configuration-id digit order.                                              */
@@ -218,8 +224,9 @@ typedef enum {
   PS_XFER_TRANSIENT = 4
 } ps_xfer_method;
 /* Host-side RNE conversion of an f32 array (canonical NaN, bit-identical to   */
-/* ps_convert): dst_type f64/f32/f16, `threads` workers (<= 1: caller's),     */
-/* simd != 0 uses F16C/AVX2 when the CPU has them.  Host pointers.            */
+/* ps_convert): dst_type f64/f32/f16/bf16, `threads` workers (<= 1: the      */
+/* caller's), simd != 0 uses F16C/AVX2 for f16/f64 when the CPU has them (bf16 */
+/* is an integer-only rounding loop).  Host pointers.                         */
 PS_API ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, int threads,
                                  int simd);
 /* One object's {type conversion then transfer} with a method (the System     */
