@@ -9,7 +9,10 @@ plain single-threaded C definition of SURVEY.md §8(a) a1-a5 (see the header of
 ``oracle.c`` for the paper passages each part follows).  Precision codes:
 0 = f64, 1 = f32, 2 = f16 (descending precision); 3 = bf16 for the
 Blackwell extension, whose buffers are raw uint16 bit
-patterns here (numpy has no bfloat16; ``widen`` gives their exact values).
+patterns here (numpy has no bfloat16; ``widen`` gives their exact values);
+4 = fp8 E4M3 and 5 = fp8 E5M2 (reading #29), raw uint8 codes whose objects
+carry a per-tensor power-of-two scale 2^k (``convert_scaled``,
+``run_config(..., with_scales=True)``).
 """
 from __future__ import annotations
 
@@ -25,8 +28,11 @@ _SRC = os.path.join(_HERE, "oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared", "-std=c11", "-Wall"]
 
-F64, F32, F16, BF16 = 0, 1, 2, 3
-NP_DTYPE = {F64: np.float64, F32: np.float32, F16: np.float16, BF16: np.uint16}
+F64, F32, F16, BF16, E4M3, E5M2 = 0, 1, 2, 3, 4, 5
+NP_DTYPE = {F64: np.float64, F32: np.float32, F16: np.float16, BF16: np.uint16,
+            E4M3: np.uint8, E5M2: np.uint8}
+FP8 = (E4M3, E5M2)
+FP8_MAX = {E4M3: 448.0, E5M2: 57344.0}
 ROWDOT_LANES = 32
 COLSUM_CHUNK = 256
 
@@ -70,6 +76,16 @@ def lib():
                                          ctypes.c_int, ctypes.c_size_t]
             L.oracle_quality.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p,
                                          ctypes.c_size_t, ctypes.POINTER(QualityResult)]
+            L.oracle_fp8_scale_exp.argtypes = [ctypes.c_double, ctypes.c_int]
+            L.oracle_convert_scaled.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p,
+                                                ctypes.c_int, ctypes.c_size_t,
+                                                ctypes.POINTER(ctypes.c_int)]
+            L.oracle_run_config_k.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_int64),
+                                              ctypes.c_int, ctypes.POINTER(ctypes.c_double),
+                                              ctypes.POINTER(ctypes.c_int),
+                                              ctypes.POINTER(ctypes.c_void_p),
+                                              ctypes.POINTER(ctypes.c_void_p),
+                                              ctypes.POINTER(ctypes.c_int)]
             L.oracle_config_decode.argtypes = [ctypes.c_int, ctypes.c_uint64,
                                                ctypes.POINTER(ctypes.c_int)]
             L.oracle_config_encode.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_int),
@@ -114,6 +130,22 @@ def convert(a: np.ndarray, src: int, dst: int) -> np.ndarray:
     if lib().oracle_convert(_ptr(a), src, _ptr(out), dst, a.size):
         raise ValueError("oracle_convert failed")
     return out
+
+
+def fp8_scale_exp(amax: float, t: int) -> int:
+    """Reading #29: smallest k in [-126, 126] with amax <= FMAX * 2^k."""
+    return int(lib().oracle_fp8_scale_exp(float(amax), t))
+
+
+def convert_scaled(a: np.ndarray, src: int, dst: int, k: int = 0):
+    """Scaled conversion (reading #29).  To fp8: returns (codes, k) with k from
+    the finite values of a.  From fp8: returns (values, k) decoding with scale 2^k."""
+    a = np.ascontiguousarray(a)
+    out = np.empty(a.shape, dtype=NP_DTYPE[dst])
+    kk = ctypes.c_int(int(k))
+    if lib().oracle_convert_scaled(_ptr(a), src, _ptr(out), dst, a.size, ctypes.byref(kk)):
+        raise ValueError("oracle_convert_scaled failed")
+    return out, int(kk.value)
 
 
 def widen(a: np.ndarray, t: int) -> np.ndarray:
@@ -184,8 +216,10 @@ def _inputs(objs, inputs):
     return arr, keep
 
 
-def run_config(kind: str, dims, prec, inputs, scalars=None) -> list:
-    """a2 + a3: final contents of every object in its assigned precision."""
+def run_config(kind: str, dims, prec, inputs, scalars=None, with_scales: bool = False):
+    """a2 + a3: final contents of every object in its assigned precision (fp8:
+    raw codes).  with_scales: also return the list of final scale exponents k
+    (None for non-fp8 objects)."""
     objs = app_objects(kind, dims)
     assert len(prec) == len(objs)
     d, nd = _dims(dims)
@@ -193,9 +227,19 @@ def run_config(kind: str, dims, prec, inputs, scalars=None) -> list:
     finals = [np.empty((o["rows"], o["cols"]), dtype=NP_DTYPE[p]) for o, p in zip(objs, prec)]
     fin = (ctypes.c_void_p * len(objs))(*[f.ctypes.data for f in finals])
     pr = (ctypes.c_int * len(prec))(*prec)
-    if lib().oracle_run_config(kind.encode(), d, nd, _scalars(scalars), pr, ins, fin):
+    ks = (ctypes.c_int * len(prec))()
+    if lib().oracle_run_config_k(kind.encode(), d, nd, _scalars(scalars), pr, ins, fin, ks):
         raise ValueError("oracle_run_config failed")
+    if with_scales:
+        return finals, [int(ks[m]) if p in FP8 else None for m, p in enumerate(prec)]
     return finals
+
+
+def values(final: np.ndarray, t: int, k=None) -> np.ndarray:
+    """Exact float64 values of an object's final contents (fp8: code * 2^k)."""
+    if t in FP8:
+        return np.ldexp(widen(final, t), int(k))
+    return widen(final, t)
 
 
 def reference(kind: str, dims, inputs, scalars=None) -> list:

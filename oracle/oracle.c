@@ -9,6 +9,10 @@
  * IEEE double).  Every narrowing conversion goes through the software
  * bit-manipulation converter below, never an FPU conversion instruction.
  *
+ * Precision codes: 0 f64, 1 f32, 2 f16 (the paper's), 3 bf16, 4 fp8
+ * E4M3, 5 fp8 E5M2 (Blackwell extensions, DESIGN.md
+ * readings #28/#29; fp8 objects carry a per-tensor power-of-two scale).
+ *
  * What it computes (readings listed in DESIGN.md):
  *   a1 config decode   ("(1+#Conv_Types)^N", order P:293)
  *   a2 input conversion of every memory object to its assigned precision
@@ -33,9 +37,14 @@
 /* c-1: software IEEE-754 converter                                      */
 /* ===================================================================== */
 
-typedef struct { int ebits, mbits, bias; } fmt_t;
-/* index = precision code: f64, f32, f16, bf16 (8 exponent, 7 fraction bits) */
-static const fmt_t FMT[4] = { {11, 52, 1023}, {8, 23, 127}, {5, 10, 15}, {8, 7, 127} };
+typedef struct { int ebits, mbits, bias, has_inf; } fmt_t;
+/* index = precision code: f64, f32, f16, bf16 (8 exponent, 7 fraction bits),
+ * fp8 E4M3 and E5M2 (reading #29).  E4M3 (OCP "fn" variant) has no infinity:
+ * its all-ones exponent field is an ordinary binade except fraction 111 = NaN,
+ * so its largest finite value is 1.75 * 2^8 = 448; a rounded magnitude above
+ * 448 (or an infinite input) becomes NaN.  E5M2 is IEEE-like (max 57344, inf). */
+static const fmt_t FMT[6] = { {11, 52, 1023, 1}, {8, 23, 127, 1}, {5, 10, 15, 1}, {8, 7, 127, 1},
+                              {4, 3, 7, 0}, {5, 2, 15, 1} };
 
 /* number of significant bits of v (0 for v == 0) */
 static int bitlen64(uint64_t v) { return v ? 64 - __builtin_clzll(v) : 0; }
@@ -57,9 +66,10 @@ uint64_t oracle_convert_bits(uint64_t x, int st, int dt) {
   uint64_t S, K;
   int xexp, E, q, r, emin_d;
 
-  /* step 2: inf / NaN */
-  if (e == emax_s) {
-    if (f == 0) return dsign | (emax_d << d->mbits);
+  /* step 2: inf / NaN (E4M3 source: only fraction all-ones is NaN, the rest of
+   * its top binade is finite; E4M3 destination: no infinity, inf -> NaN) */
+  if (e == emax_s && (s->has_inf || f == (1ull << s->mbits) - 1)) {
+    if (f == 0 && s->has_inf) return d->has_inf ? (dsign | (emax_d << d->mbits)) : canonical_nan(d);
     return canonical_nan(d);
   }
   /* step 3: signed zero */
@@ -88,16 +98,24 @@ uint64_t oracle_convert_bits(uint64_t x, int st, int dt) {
   if (K >= (1ull << d->mbits)) {
     int64_t biased = (int64_t)q + d->mbits + d->bias;
     if (K == (1ull << (d->mbits + 1))) { K >>= 1; biased++; }
+    if (!d->has_inf) {   /* E4M3: the top binade is finite up to fraction 110 */
+      if (biased > (int64_t)emax_d || (biased == (int64_t)emax_d && K == (1ull << (d->mbits + 1)) - 1))
+        return canonical_nan(d);                                           /* overflow -> NaN */
+      return dsign | ((uint64_t)biased << d->mbits) | (K - (1ull << d->mbits));
+    }
     if (biased >= (int64_t)emax_d) return dsign | (emax_d << d->mbits);   /* overflow -> inf */
     return dsign | ((uint64_t)biased << d->mbits) | (K - (1ull << d->mbits));
   }
   return dsign | K;                /* subnormal (q == emin_d - mbits) */
 }
 
+static int is_fp8(int t) { return t == OR_E4M3 || t == OR_E5M2; }
+
 static uint64_t load_bits(const void *p, int t, size_t i) {
   switch (t) {
     case OR_F64: { uint64_t b; memcpy(&b, (const char *)p + 8 * i, 8); return b; }
     case OR_F32: { uint32_t b; memcpy(&b, (const char *)p + 4 * i, 4); return b; }
+    case OR_E4M3: case OR_E5M2: return ((const uint8_t *)p)[i];
     default:     { uint16_t b; memcpy(&b, (const char *)p + 2 * i, 2); return b; }
   }
 }
@@ -105,13 +123,14 @@ static void store_bits(void *p, int t, size_t i, uint64_t b) {
   switch (t) {
     case OR_F64: memcpy((char *)p + 8 * i, &b, 8); break;
     case OR_F32: { uint32_t v = (uint32_t)b; memcpy((char *)p + 4 * i, &v, 4); break; }
+    case OR_E4M3: case OR_E5M2: ((uint8_t *)p)[i] = (uint8_t)b; break;
     default:     { uint16_t v = (uint16_t)b; memcpy((char *)p + 2 * i, &v, 2); break; }
   }
 }
 
 int oracle_convert(const void *src, int st, void *dst, int dt, size_t n) {
   size_t i;
-  if (st < 0 || st > 3 || dt < 0 || dt > 3) return 1;
+  if (st < 0 || st > 5 || dt < 0 || dt > 5) return 1;
   if (n && (!src || !dst)) return 1;
   for (i = 0; i < n; i++) {
     uint64_t b = load_bits(src, st, i);
@@ -125,10 +144,59 @@ static uint64_t double_to_bits(double d) { uint64_t b; memcpy(&b, &d, 8); return
 static uint32_t float_to_bits(float f) { uint32_t b; memcpy(&b, &f, 4); return b; }
 static float bits_to_float(uint32_t b) { float f; memcpy(&f, &b, 4); return f; }
 
-/* exact widening of element i of a buffer of type t to double */
+/* exact widening of element i of a buffer of type t to double (fp8: the code's
+ * own value, without the object's scale) */
 static double widen(const void *p, int t, size_t i) {
   uint64_t b = load_bits(p, t, i);
   return bits_to_double(t == OR_F64 ? b : oracle_convert_bits(b, t, OR_F64));
+}
+
+/* ---- fp8 per-tensor power-of-two scale (reading #29) ------------------- */
+static double fp8_max(int t) { return t == OR_E4M3 ? 448.0 : 57344.0; }
+
+int oracle_fp8_scale_exp(double amax, int t) {
+  int k;
+  if (!(amax > 0.0)) return 0;
+  for (k = ORACLE_FP8_KMIN; k <= ORACLE_FP8_KMAX; k++)
+    if (amax <= ldexp(fp8_max(t), k)) return k;   /* ldexp: exact power-of-two scaling */
+  return ORACLE_FP8_KMAX;
+}
+/* q = RNE_fp8(v * 2^-k): the product is exact in double (or, below 2^-1022,
+ * far under half the smallest fp8 subnormal, so the code is +-0 either way) */
+static uint64_t fp8_encode(double v, int k, int t) {
+  return oracle_convert_bits(double_to_bits(ldexp(v, -k)), OR_F64, t);
+}
+static double fp8_decode(uint64_t q, int k, int t) {
+  return ldexp(bits_to_double(oracle_convert_bits(q, t, OR_F64)), k);
+}
+
+int oracle_convert_scaled(const void *src, int st, void *dst, int dt, size_t n, int *k_io) {
+  size_t i;
+  double amax = 0.0;
+  int k;
+  if (st < 0 || st > 5 || dt < 0 || dt > 5) return 1;
+  if (n && (!src || !dst)) return 1;
+  if (!is_fp8(st) && !is_fp8(dt)) return oracle_convert(src, st, dst, dt, n);
+  if (!k_io) return 1;
+  if (!is_fp8(dt)) {                         /* decode: RNE_dst(q * 2^k) */
+    for (i = 0; i < n; i++) {
+      double v = fp8_decode(load_bits(src, st, i), *k_io, st);
+      store_bits(dst, dt, i, dt == OR_F64 ? double_to_bits(v)
+                                          : oracle_convert_bits(double_to_bits(v), OR_F64, dt));
+    }
+    return 0;
+  }
+  for (i = 0; i < n; i++) {                  /* amax over the finite source values */
+    double v = is_fp8(st) ? fp8_decode(load_bits(src, st, i), *k_io, st) : widen(src, st, i);
+    if (isfinite(v) && fabs(v) > amax) amax = fabs(v);
+  }
+  k = oracle_fp8_scale_exp(amax, dt);
+  for (i = 0; i < n; i++) {
+    double v = is_fp8(st) ? fp8_decode(load_bits(src, st, i), *k_io, st) : widen(src, st, i);
+    store_bits(dst, dt, i, fp8_encode(v, k, dt));
+  }
+  *k_io = k;
+  return 0;
 }
 
 /* ===================================================================== */
@@ -153,7 +221,7 @@ int oracle_quality(const void *out, int ot, const double *ref, size_t n,
                    oracle_quality_result *res) {
   double s = 0.0, mx = 0.0;
   uint64_t nf = 0;
-  if (!res || ot < 0 || ot > 3) return 1;
+  if (!res || ot < 0 || ot > 5) return 1;
   oracle_quality_accumulate(out, ot, ref, n, &s, &mx, &nf);
   res->n = n;
   res->mean_rel = n ? s / (double)n : 0.0;
@@ -171,7 +239,7 @@ int oracle_quality(const void *out, int ot, const double *ref, size_t n,
 int oracle_config_decode_radix(int m, int radix, uint64_t id, int *prec) {
   int i;
   uint64_t space = 1;
-  if (radix != 3 && radix != 4) return 1;
+  if (radix != 3 && radix != 4 && radix != 6) return 1;
   for (i = 0; i < m; i++) space *= (uint64_t)radix;
   if (m <= 0 || id >= space || !prec) return 1;
   for (i = 0; i < m; i++) { prec[i] = (int)(id % (uint64_t)radix); id /= (uint64_t)radix; }
@@ -181,7 +249,7 @@ int oracle_config_decode_radix(int m, int radix, uint64_t id, int *prec) {
 int oracle_config_encode_radix(int m, int radix, const int *prec, uint64_t *id) {
   int i;
   uint64_t v = 0, w = 1;
-  if (m <= 0 || !prec || !id || (radix != 3 && radix != 4)) return 1;
+  if (m <= 0 || !prec || !id || (radix != 3 && radix != 4 && radix != 6)) return 1;
   for (i = 0; i < m; i++) {
     if (prec[i] < 0 || prec[i] >= radix) return 1;
     v += (uint64_t)prec[i] * w;
@@ -201,12 +269,17 @@ int oracle_config_encode(int m, const int *prec, uint64_t *id) { return oracle_c
 /* An object stored in precision `type`.  In sampling mode (oracle_sample) an
  * input object may instead be "lazy": element i is RNE_type(src[i]) converted
  * on access from the original f32 data -- the same value a2 would have stored. */
-typedef struct { int type; size_t n; void *p; const float *src; } obj_t;
+/* An fp8 object (reading #29) also keeps val[i] = the exact current value
+ * q_i * 2^k of every element, its scale exponent k, and a dirty flag: stores
+ * inside a statement go to val; fp8_commit() at the end of every statement that
+ * wrote the object re-quantises the whole object with a fresh per-tensor scale. */
+typedef struct { int type; size_t n; void *p; const float *src; double *val; int k, dirty; } obj_t;
 
-static size_t tsize(int t) { return t == OR_F64 ? 8 : (t == OR_F32 ? 4 : 2); }
+static size_t tsize(int t) { return t == OR_F64 ? 8 : (t == OR_F32 ? 4 : (is_fp8(t) ? 1 : 2)); }
 
 /* R1: load = exact widening of the stored element */
 static double ld(const obj_t *o, size_t i) {
+  if (o->val) return o->val[i];              /* fp8: q_i * 2^k (or this statement's store) */
   if (o->src) {
     uint32_t b;
     memcpy(&b, &o->src[i], 4);
@@ -220,6 +293,11 @@ static double ld(const obj_t *o, size_t i) {
  * value v is exactly representable in T. */
 static void st(obj_t *o, size_t i, double v, int T) {
   uint64_t b;
+  if (o->val) {                              /* fp8: keep the value in T until the commit */
+    o->val[i] = (T == OR_F64) ? v : (double)(float)v;
+    o->dirty = 1;
+    return;
+  }
   if (o->type == OR_F64) { ((double *)o->p)[i] = v; return; }
   if (T == OR_F64) b = oracle_convert_bits(double_to_bits(v), OR_F64, o->type);
   else if (o->type == OR_F32) b = float_to_bits((float)v);        /* exact: v is f32 */
@@ -227,8 +305,25 @@ static void st(obj_t *o, size_t i, double v, int T) {
   store_bits(o->p, o->type, i, b);
 }
 
-/* R2: T = widest of the touched objects, floored at f32 (code 0 = widest; f16 and
- * bf16, codes 2 and 3, are both narrower than f32, so they compute in f32) */
+/* Reading #29: end of a statement that wrote fp8 object o -- amax over its
+ * finite values, k, then every element re-encoded as RNE_fp8(v * 2^-k). */
+static void fp8_commit(obj_t *o) {
+  size_t i;
+  double amax = 0.0;
+  if (!o->val || !o->dirty) return;
+  for (i = 0; i < o->n; i++)
+    if (isfinite(o->val[i]) && fabs(o->val[i]) > amax) amax = fabs(o->val[i]);
+  o->k = oracle_fp8_scale_exp(amax, o->type);
+  for (i = 0; i < o->n; i++) {
+    uint64_t q = fp8_encode(o->val[i], o->k, o->type);
+    store_bits(o->p, o->type, i, q);
+    o->val[i] = fp8_decode(q, o->k, o->type);
+  }
+  o->dirty = 0;
+}
+
+/* R2: T = widest of the touched objects, floored at f32 (code 0 = widest; f16,
+ * bf16, e4m3 and e5m2, codes 2-5, are all narrower than f32, so they compute in f32) */
 static int W2(int a, int b) { int t = a < b ? a : b; return t < OR_F32 ? t : OR_F32; }
 static int W3(int a, int b, int c) { return W2(W2(a, b), c); }
 
@@ -282,7 +377,9 @@ static double dot_chain(int T, const obj_t *A, size_t ai, size_t ask,
  *  - row: tile sums added left to right. */
 static double rowdot(int T, const obj_t *A, size_t row0, size_t n, const obj_t *x) {
   double lane[ORACLE_ROWDOT_LANES], nxt[ORACLE_ROWDOT_LANES];
-  size_t V = 16 / tsize(A->type), W = ORACLE_ROWDOT_LANES * V;
+  /* an fp8 matrix is decoded into T before the statement (reading #29), so its
+   * lane chunk is that of T */
+  size_t V = 16 / (is_fp8(A->type) ? tsize(T) : tsize(A->type)), W = ORACLE_ROWDOT_LANES * V;
   size_t nslab = (n + W - 1) / W, s, v;
   double total = 0.0, tile = 0.0;
   int l, off;
@@ -477,6 +574,7 @@ static void app_gemm(obj_t *o, const int64_t *d, const double *sc) {
       double bc = t_mul(T, be, ld(&o[2], i * NJ + j));
       st(&o[2], i * NJ + j, t_fma(T, al, acc, bc), T);
     }
+  fp8_commit(&o[2]);
 }
 
 /* out[i][j] <- sum_k A[i][k] B[k][j] (no epilogue), R3 order */
@@ -485,6 +583,7 @@ static void matmul(obj_t *A, obj_t *B, obj_t *C, size_t NI, size_t NJ, size_t NK
   int T = W3(A->type, B->type, C->type);
   for (i = 0; i < NI; i++)
     for (j = 0; j < NJ; j++) st(C, i * NJ + j, dot_chain(T, A, i * NK, 1, B, j, NJ, NK), T);
+  fp8_commit(C);
 }
 
 static void app_2mm(obj_t *o, const int64_t *d) {
@@ -504,14 +603,18 @@ static void app_atax(obj_t *o, const int64_t *d) {
   size_t NX = d[0], NY = d[1], i, j;
   int T1 = W3(o[0].type, o[1].type, o[3].type), T2 = W3(o[0].type, o[3].type, o[2].type);
   for (i = 0; i < NX; i++) st(&o[3], i, rowdot(T1, &o[0], i * NY, NY, &o[1]), T1);  /* tmp <- A x */
+  fp8_commit(&o[3]);
   for (j = 0; j < NY; j++) st(&o[2], j, colsum(T2, &o[0], NX, NY, j, &o[3], 0), T2); /* y <- A^T tmp */
+  fp8_commit(&o[2]);
 }
 
 static void app_bicg(obj_t *o, const int64_t *d) {
   size_t NX = d[0], NY = d[1], i, j;
   int T1 = W3(o[0].type, o[1].type, o[2].type), T2 = W3(o[0].type, o[3].type, o[4].type);
   for (j = 0; j < NY; j++) st(&o[2], j, colsum(T1, &o[0], NX, NY, j, &o[1], 0), T1); /* s <- A^T r */
+  fp8_commit(&o[2]);
   for (i = 0; i < NX; i++) st(&o[4], i, rowdot(T2, &o[0], i * NY, NY, &o[3]), T2);  /* q <- A p */
+  fp8_commit(&o[4]);
 }
 
 static void app_gesummv(obj_t *o, const int64_t *d, const double *sc) {
@@ -521,9 +624,12 @@ static void app_gesummv(obj_t *o, const int64_t *d, const double *sc) {
   int T3 = W2(o[4].type, o[3].type);              /* y   <- alpha tmp + beta y */
   double al = t_lit(T3, scalar_or(sc, 0, 43532.0)), be = t_lit(T3, scalar_or(sc, 1, 12313.0));
   for (i = 0; i < N; i++) st(&o[4], i, rowdot(T1, &o[0], i * N, N, &o[2]), T1);
+  fp8_commit(&o[4]);
   for (i = 0; i < N; i++) st(&o[3], i, rowdot(T2, &o[1], i * N, N, &o[2]), T2);
+  fp8_commit(&o[3]);
   for (i = 0; i < N; i++)
     st(&o[3], i, t_fma(T3, al, ld(&o[4], i), t_mul(T3, be, ld(&o[3], i))), T3);
+  fp8_commit(&o[3]);
 }
 
 /* symmetric product sym[j1][j2] = sym[j2][j1] = sum_i X_ij1 X_ij2 (R3),
@@ -541,6 +647,7 @@ static void syrk_upper(obj_t *X, obj_t *S, size_t N, size_t M, int diag_one, dou
       st(S, j2 * M + j1, acc, T);
     }
   }
+  fp8_commit(S);
 }
 
 static void col_mean(obj_t *data, obj_t *mean, size_t N, size_t M) {
@@ -548,6 +655,7 @@ static void col_mean(obj_t *data, obj_t *mean, size_t N, size_t M) {
   int T = W2(data->type, mean->type);
   double n = t_lit(T, (double)N);
   for (j = 0; j < M; j++) st(mean, j, t_div(T, colsum(T, data, N, M, j, NULL, 1), n), T);
+  fp8_commit(mean);
 }
 
 static void app_corr(obj_t *o, const int64_t *d, const double *sc) {
@@ -560,11 +668,13 @@ static void app_corr(obj_t *o, const int64_t *d, const double *sc) {
     double s = t_sqrt(T2, t_div(T2, colsum(T2, &o[0], N, M, j, &o[1], 2), n2));
     st(&o[2], j, s <= eps ? 1.0 : s, T2);
   }
+  fp8_commit(&o[2]);
   for (i = 0; i < N; i++)                                         /* normalise */
     for (j = 0; j < M; j++) {
       double dd = t_sub(T3, ld(&o[0], i * M + j), ld(&o[1], j));
       st(&o[0], i * M + j, t_div(T3, dd, t_mul(T3, sqn, ld(&o[2], j))), T3);
     }
+  fp8_commit(&o[0]);
   syrk_upper(&o[0], &o[3], N, M, 1, 0.0);                         /* symmat */
 }
 
@@ -575,6 +685,7 @@ static void app_covar(obj_t *o, const int64_t *d) {
   for (i = 0; i < N; i++)                                         /* centre */
     for (j = 0; j < M; j++)
       st(&o[0], i * M + j, t_sub(T2, ld(&o[0], i * M + j), ld(&o[1], j)), T2);
+  fp8_commit(&o[0]);
   syrk_upper(&o[0], &o[2], N, M, 0, (double)N - 1.0);             /* symmat */
 }
 
@@ -584,8 +695,10 @@ static void app_mvt(obj_t *o, const int64_t *d) {
   int T1 = W3(o[0].type, o[1].type, o[3].type), T2 = W3(o[0].type, o[2].type, o[4].type);
   for (i = 0; i < N; i++)
     st(&o[1], i, t_add(T1, ld(&o[1], i), rowdot(T1, &o[0], i * N, N, &o[3])), T1);
+  fp8_commit(&o[1]);
   for (i = 0; i < N; i++)
     st(&o[2], i, t_add(T2, ld(&o[2], i), colsum(T2, &o[0], N, N, i, &o[4], 0)), T2);
+  fp8_commit(&o[2]);
 }
 
 /* SYRK (BLAS 'T' form, reading #23): C <- alpha A^T A + beta C over A: N x M,
@@ -601,6 +714,7 @@ static void app_syrk(obj_t *o, const int64_t *d, const double *sc) {
       st(&o[1], j1 * M + j2, r, T);
       st(&o[1], j2 * M + j1, r, T);
     }
+  fp8_commit(&o[1]);
 }
 
 /* 2DCONV (reading #24): B_ij = c11 A(i-1,j-1) + c12 A(i,j-1) + c13 A(i+1,j-1)
@@ -627,6 +741,7 @@ static void app_conv2d(obj_t *o, const int64_t *d) {
       int border = (i == 0 || j == 0 || i + 1 >= NI || j + 1 >= NJ);
       st(&o[1], i * NJ + j, border ? 0.0 : conv2d_at(T, &o[0], NJ, i, j), T);
     }
+  fp8_commit(&o[1]);
 }
 
 /* SYR2K (BLAS 'T' form, reading #25): C <- alpha A^T B + beta C ; C <- alpha B^T A + C
@@ -640,11 +755,13 @@ static void app_syr2k(obj_t *o, const int64_t *d, const double *sc) {
       double s1 = dot_chain(T, &o[0], i, M, &o[1], j, M, N);
       st(&o[2], i * M + j, t_fma(T, al, s1, t_mul(T, be, ld(&o[2], i * M + j))), T);
     }
+  fp8_commit(&o[2]);
   for (i = 0; i < M; i++)
     for (j = 0; j < M; j++) {
       double s2 = dot_chain(T, &o[1], i, M, &o[0], j, M, N);
       st(&o[2], i * M + j, t_fma(T, al, s2, ld(&o[2], i * M + j)), T);
     }
+  fp8_commit(&o[2]);
 }
 
 /* 3DCONV (reading #26): 27-point stencil on A[NI][NJ][NK]: the 2DCONV weights on
@@ -674,6 +791,7 @@ static void app_conv3d(obj_t *o, const int64_t *d) {
         int border = i == 0 || j == 0 || k == 0 || i + 1 >= NI || j + 1 >= NJ || k + 1 >= NK;
         st(&o[1], (i * NJ + j) * NK + k, border ? 0.0 : conv3d_at(T, &o[0], NJ, NK, i, j, k), T);
       }
+  fp8_commit(&o[1]);
 }
 
 /* FDTD-2D (reading #27), TMAX steps over ex, ey, hz (NX x NY), each statement a
@@ -695,11 +813,13 @@ static void app_fdtd2d(obj_t *o, const int64_t *d) {
         double dh = t_sub(T2, ld(&o[3], i * NY + j), ld(&o[3], (i - 1) * NY + j));
         st(&o[2], i * NY + j, t_sub(T2, ld(&o[2], i * NY + j), t_mul(T2, h2, dh)), T2);
       }
+    fp8_commit(&o[2]);   /* the ey statement = row 0 from fict + the update of rows >= 1 */
     for (i = 0; i < NX; i++)
       for (j = 1; j < NY; j++) {
         double dh = t_sub(T3, ld(&o[3], i * NY + j), ld(&o[3], i * NY + j - 1));
         st(&o[1], i * NY + j, t_sub(T3, ld(&o[1], i * NY + j), t_mul(T3, h3, dh)), T3);
       }
+    fp8_commit(&o[1]);
     for (i = 0; i + 1 < NX; i++)
       for (j = 0; j + 1 < NY; j++) {
         double s = t_sub(T4, ld(&o[1], i * NY + j + 1), ld(&o[1], i * NY + j));
@@ -707,6 +827,7 @@ static void app_fdtd2d(obj_t *o, const int64_t *d) {
         s = t_sub(T4, s, ld(&o[2], i * NY + j));
         st(&o[3], i * NY + j, t_sub(T4, ld(&o[3], i * NY + j), t_mul(T4, c4, s)), T4);
       }
+    fp8_commit(&o[3]);
   }
 }
 
@@ -730,7 +851,7 @@ static int run_objects(const app_def_t *a, const int64_t *d, const double *sc, o
 
 static void free_objects(obj_t *o, int n) {
   int m;
-  for (m = 0; m < n; m++) free(o[m].p);
+  for (m = 0; m < n; m++) { free(o[m].p); free(o[m].val); }
 }
 
 /* a2 + a3 */
@@ -744,14 +865,25 @@ static int run_to_objects(const char *kind, const int64_t *dims, int ndims, cons
   shapes(a, d, rows, cols);
   memset(o, 0, sizeof(obj_t) * 8);
   for (m = 0; m < a->nobj; m++) {
-    if (prec[m] < 0 || prec[m] > 3) { free_objects(o, m); return 1; }
+    if (prec[m] < 0 || prec[m] > 5) { free_objects(o, m); return 1; }
     o[m].type = prec[m];
     o[m].n = (size_t)(rows[m] * cols[m]);
     o[m].p = calloc(o[m].n ? o[m].n : 1, tsize(prec[m]));
     if (!o[m].p) { free_objects(o, m); return 1; }
+    if (is_fp8(prec[m])) {                              /* reading #29: values + scale */
+      o[m].val = (double *)calloc(o[m].n ? o[m].n : 1, sizeof(double));
+      if (!o[m].val) { free_objects(o, m + 1); return 1; }
+    }
     if (a->roles[m] == 0 || a->roles[m] == 2) {         /* a2: convert orig f32 -> c(m) */
       if (!inputs || !inputs[m]) { free_objects(o, m + 1); return 1; }
-      oracle_convert(inputs[m], OR_F32, o[m].p, prec[m], o[m].n);
+      if (is_fp8(prec[m])) {                            /* exact f32 values, then quantise */
+        size_t i;
+        for (i = 0; i < o[m].n; i++) o[m].val[i] = (double)inputs[m][i];
+        o[m].dirty = 1;
+        fp8_commit(&o[m]);
+      } else {
+        oracle_convert(inputs[m], OR_F32, o[m].p, prec[m], o[m].n);
+      }
     }
   }
   run_objects(a, d, sc, o);
@@ -759,17 +891,25 @@ static int run_to_objects(const char *kind, const int64_t *dims, int ndims, cons
   return 0;
 }
 
-int oracle_run_config(const char *kind, const int64_t *dims, int ndims, const double *sc,
-                      const int *prec, const float *const *inputs, void *const *finals) {
+int oracle_run_config_k(const char *kind, const int64_t *dims, int ndims, const double *sc,
+                        const int *prec, const float *const *inputs, void *const *finals,
+                        int *scale_exps) {
   obj_t o[8];
   const app_def_t *a;
   int64_t d[8];
   int m;
   if (run_to_objects(kind, dims, ndims, sc, prec, inputs, o, &a, d)) return 1;
-  for (m = 0; m < a->nobj; m++)
+  for (m = 0; m < a->nobj; m++) {
     if (finals && finals[m]) memcpy(finals[m], o[m].p, o[m].n * tsize(o[m].type));
+    if (scale_exps && is_fp8(o[m].type)) scale_exps[m] = o[m].k;
+  }
   free_objects(o, a->nobj);
   return 0;
+}
+
+int oracle_run_config(const char *kind, const int64_t *dims, int ndims, const double *sc,
+                      const int *prec, const float *const *inputs, void *const *finals) {
+  return oracle_run_config_k(kind, dims, ndims, sc, prec, inputs, finals, NULL);
 }
 
 int oracle_evaluate(const char *kind, const int64_t *dims, int ndims, const double *sc,
@@ -788,7 +928,13 @@ int oracle_evaluate(const char *kind, const int64_t *dims, int ndims, const doub
     if (!a->outputs[m]) continue;
     /* a4: back-conversion c(o) -> orig (f32) */
     buf = (delivered && delivered[m]) ? delivered[m] : (float *)malloc(o[m].n * 4 + 4);
-    oracle_convert(o[m].p, o[m].type, buf, OR_F32, o[m].n);
+    if (o[m].val) {                         /* fp8: RNE_f32(q * 2^k) */
+      size_t i;
+      for (i = 0; i < o[m].n; i++)
+        buf[i] = bits_to_float((uint32_t)oracle_convert_bits(double_to_bits(o[m].val[i]), OR_F64, OR_F32));
+    } else {
+      oracle_convert(o[m].p, o[m].type, buf, OR_F32, o[m].n);
+    }
     /* a5: quality of the delivered output vs the fp64 run */
     oracle_quality_accumulate(buf, OR_F32, ref[m], o[m].n, &s, &mx, &nf);
     n += o[m].n;
@@ -814,12 +960,12 @@ int oracle_evaluate(const char *kind, const int64_t *dims, int ndims, const doub
 
 static double round_to(int type, double v, int T) {
   unsigned char buf[8];
-  obj_t o = {type, 1, buf, NULL};
+  obj_t o = {type, 1, buf, NULL, NULL, 0, 0};
   st(&o, 0, v, T);
   return ld(&o, 0);
 }
 static obj_t new_obj(int type, size_t n) {
-  obj_t o = {type, n, calloc(n ? n : 1, tsize(type)), NULL};
+  obj_t o = {type, n, calloc(n ? n : 1, tsize(type)), NULL, NULL, 0, 0};
   return o;
 }
 
@@ -859,7 +1005,7 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
   shapes(a, d, R, C);
   memset(in, 0, sizeof(in));
   for (t = 0; t < a->nobj; t++) {
-    if (prec[t] < 0 || prec[t] > 3) return 1;
+    if (prec[t] < 0 || prec[t] > 3) return 1;   /* fp8 (per-tensor scale): not sampleable */
     in[t].type = prec[t];
     in[t].n = (size_t)(R[t] * C[t]);
     if (a->roles[t] == 0 || a->roles[t] == 2) {

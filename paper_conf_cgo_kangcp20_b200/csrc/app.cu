@@ -960,7 +960,7 @@ ps_status ps_search(ps_app *a, double toq, int repeats, void *stream, ps_search_
   std::map<uint64_t, Trial> seen;
   auto encode = [&](const int *prec) {
     uint64_t id = 0, w = 1;
-    for (int m = 0; m < M; m++) { id += (uint64_t)prec[m] * w; w *= 3; }
+    for (int m = 0; m < M; m++) { id += (uint64_t)prec[m] * w; w *= (uint64_t)radix(a); }
     return id;
   };
   // RunApp (Alg. 1 line 8): median total time of `repeats` runs; never re-run a config
