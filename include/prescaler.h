@@ -39,8 +39,12 @@ extern "C" {
 /* precision codes in the paper's descending-precision order; PS_BF16
  * is the Blackwell extension (reading #28): raw
  * uint16 bit patterns (1 sign, 8 exponent, 7 fraction bits), RNE narrowing with
- * subnormals, overflow to inf, canonical NaN 0x7FFF. */
-typedef enum { PS_F64 = 0, PS_F32 = 1, PS_F16 = 2, PS_BF16 = 3 } ps_dtype;
+ * subnormals, overflow to inf, canonical NaN 0x7FFF.  PS_E4M3 / PS_E5M2 are the
+ * fp8 extensions (reading #29): raw uint8 codes, OCP E4M3 "fn" (bias 7, no inf,
+ * NaN 0x7F, max 448; overflow -> NaN) and E5M2 (bias 15, max 57344, overflow ->
+ * inf), canonical NaN 0x7F; an fp8 memory object carries a per-tensor power-of-
+ * two scale (ps_fp8_scale). */
+typedef enum { PS_F64 = 0, PS_F32 = 1, PS_F16 = 2, PS_BF16 = 3, PS_E4M3 = 4, PS_E5M2 = 5 } ps_dtype;
 
 typedef enum {
   PS_OK = 0,
@@ -71,8 +75,29 @@ PS_API uint64_t ps_kernel_launches(void);
 /*   pointers, any alignment (16-byte aligned pointers take the vector path);    */
 /*   overlapping ranges -> PS_ERR_INVALID; n == 0 is a no-op; src_type ==        */
 /*   dst_type is a device-to-device copy.  Asynchronous on `stream`.             */
+/*   fp8 types are converted UNSCALED here (scale 2^0); see ps_convert_scaled. */
 PS_API ps_status ps_convert(const void *src, int src_type, void *dst, int dst_type, size_t n,
                      void *stream);
+
+/* Per-tensor power-of-two scale of an fp8 memory object (reading #29).  A
+ * 16-byte record in DEVICE memory, caller-owned: element i of the object holds
+ * code q_i with value q_i * 2^k. */
+typedef struct {
+  uint64_t amax_bits;  /* scratch: IEEE f64 bits of the last amax (library-written) */
+  int32_t k;           /* scale exponent, in [-126, 126]                             */
+  int32_t reserved;
+} ps_fp8_scale;
+/* Scaled conversion of an fp8 memory object (reading #29):
+ *   dst_type fp8, src_type f64/f32/f16/bf16: amax = max |src| over the finite
+ *     elements; k = the smallest integer in [-126, 126] with amax <= FMAX * 2^k
+ *     (FMAX 448 / 57344; k = 0 if amax == 0; 126 if none); dst[i] =
+ *     RNE_fp8(src[i] * 2^-k) in one rounding; writes scale->k (and amax_bits);
+ *   src_type fp8, dst_type f64/f32/f16/bf16: dst[i] = RNE_dst(q_i * 2^scale->k);
+ *   fp8 -> fp8 and non-fp8 pairs: PS_ERR_UNSUPPORTED / use ps_convert.
+ *   scale: device pointer (16-byte record); src, dst as in ps_convert.
+ *   Asynchronous on `stream` (two kernels: amax, then encode). */
+PS_API ps_status ps_convert_scaled(const void *src, int src_type, void *dst, int dst_type, size_t n,
+                            ps_fp8_scale *scale, void *stream);
 
 /* ------------------------------------------------------------------------- */
 /* (2) Output quality of one buffer against the fp64 run (reading #7):   */
@@ -127,6 +152,11 @@ PS_API ps_status ps_app_object_info(const ps_app *app, int m, ps_object_info *ou
 /* least significant); without it the space is the paper's 3^M.               */
 #define PS_FLAG_NO_TENSOR_CORES 1u
 #define PS_FLAG_BF16 2u
+/* PS_FLAG_FP8 extends the alphabet to {f64, f32, f16, bf16, e4m3, e5m2}: ids run */
+/* over 6^M (radix 6).  fp8 objects carry a per-tensor scale (reading #29); the   */
+/* workspace then also holds one n*8-byte staging region per object, so set the   */
+/* flags BEFORE ps_app_workspace_bytes / ps_app_bind.                             */
+#define PS_FLAG_FP8 4u
 PS_API ps_status ps_app_set_flags(ps_app *app, uint32_t flags);
 /* Device workspace the caller must allocate (>= 256-byte aligned). */
 PS_API size_t ps_app_workspace_bytes(const ps_app *app);

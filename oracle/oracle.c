@@ -808,12 +808,13 @@ static void app_fdtd2d(obj_t *o, const int64_t *d) {
   double h2 = t_lit(T2, 0.5), h3 = t_lit(T3, 0.5), c4 = t_lit(T4, 0.7);
   for (t = 0; t < TM; t++) {
     for (j = 0; j < NY; j++) st(&o[2], j, ld(&o[0], t), T1);
+    fp8_commit(&o[2]);   /* ey[0][j] = fict[t] is its own statement (reading #29) */
     for (i = 1; i < NX; i++)
       for (j = 0; j < NY; j++) {
         double dh = t_sub(T2, ld(&o[3], i * NY + j), ld(&o[3], (i - 1) * NY + j));
         st(&o[2], i * NY + j, t_sub(T2, ld(&o[2], i * NY + j), t_mul(T2, h2, dh)), T2);
       }
-    fp8_commit(&o[2]);   /* the ey statement = row 0 from fict + the update of rows >= 1 */
+    fp8_commit(&o[2]);
     for (i = 0; i < NX; i++)
       for (j = 1; j < NY; j++) {
         double dh = t_sub(T3, ld(&o[3], i * NY + j), ld(&o[3], i * NY + j - 1));

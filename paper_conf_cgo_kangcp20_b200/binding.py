@@ -18,15 +18,17 @@ LIB_PATH = os.path.join(HERE, "libprescaler.so")
 
 F64, F32, F16 = 0, 1, 2                      # ps_dtype (descending precision)
 BF16 = 3                                     # Blackwell extension (reading #28)
+E4M3, E5M2 = 4, 5                            # fp8 objects with a per-tensor scale (reading #29)
 METRIC_MRE, METRIC_MAX_REL = 0, 1
 FLAG_NO_TENSOR_CORES = 1
 FLAG_BF16 = 2                                # configuration alphabet {f64, f32, f16, bf16}: 4^M
+FLAG_FP8 = 4                                 # + e4m3, e5m2: 6^M (set before bind)
 ROLE_IN, ROLE_OUT, ROLE_INOUT, ROLE_TEMP = 0, 1, 2, 3
 
 # every symbol include/prescaler.h declares
 SYMBOLS = [
     "ps_status_string", "ps_last_error", "ps_version", "ps_kernel_launches", "ps_convert",
-    "ps_quality",
+    "ps_convert_scaled", "ps_quality",
     "ps_app_create", "ps_app_destroy", "ps_app_num_objects", "ps_app_object_info",
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
@@ -96,6 +98,8 @@ def lib():
                 "ps_version": (ctypes.c_char_p, []),
                 "ps_kernel_launches": (ctypes.c_uint64, []),
                 "ps_convert": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_int, ctypes.c_size_t, vp]),
+                "ps_convert_scaled": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_int, ctypes.c_size_t,
+                                                     vp, vp]),
                 "ps_quality": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_size_t, ctypes.c_int, vp,
                                               ctypes.POINTER(PsQualityResult)]),
                 "ps_app_create": (ctypes.c_int, [ctypes.c_char_p, i64p, ctypes.c_int,
@@ -180,7 +184,8 @@ def _stream(stream):
 
 def torch_dtype(code: int):
     import torch
-    return {F64: torch.float64, F32: torch.float32, F16: torch.float16}[code]
+    return {F64: torch.float64, F32: torch.float32, F16: torch.float16, BF16: torch.bfloat16,
+            E4M3: torch.uint8, E5M2: torch.uint8}[code]
 
 
 # -------------------------------------------------------------- (1) convert
@@ -192,11 +197,23 @@ def ps_convert(src, src_type: int, dst, dst_type: int, n: int = None, stream=Non
            "ps_convert")
 
 
+def ps_convert_scaled(src, src_type: int, dst, dst_type: int, scale, n: int = None,
+                      stream=None) -> None:
+    """fp8 object conversion with a per-tensor power-of-two scale (reading #29).
+    scale: a 16-byte device buffer (ps_fp8_scale: u64 amax bits, i32 k, i32 pad);
+    to fp8 it receives k, from fp8 it supplies k."""
+    if n is None:
+        n = src.numel()
+    _check(lib().ps_convert_scaled(_ptr(src), src_type, _ptr(dst), dst_type, n, _ptr(scale),
+                                   _stream(stream)), "ps_convert_scaled")
+
+
 def ps_host_convert(src: np.ndarray, dst_type: int, threads: int = 0, simd: bool = True) -> np.ndarray:
     """Host-side RNE conversion of an f32 numpy array (Fig. 3a: simd=False, threads=1;
     Fig. 3b: SIMD + threads).  Bit-identical to ps_convert."""
     src = np.ascontiguousarray(src, dtype=np.float32)
-    out = np.empty(src.shape, dtype={F64: np.float64, F32: np.float32, F16: np.float16}[dst_type])
+    out = np.empty(src.shape, dtype={F64: np.float64, F32: np.float32, F16: np.float16,
+                                     BF16: np.uint16}[dst_type])
     _check(lib().ps_host_convert(src.ctypes.data, out.ctypes.data, dst_type, src.size, threads,
                                  1 if simd else 0), "ps_host_convert")
     return out
@@ -260,15 +277,17 @@ class App:
 
     @property
     def radix(self) -> int:
-        return 4 if self.flags & FLAG_BF16 else 3
+        return 6 if self.flags & FLAG_FP8 else (4 if self.flags & FLAG_BF16 else 3)
 
     @property
     def space(self) -> int:
         return self.radix ** self.num_objects
 
     def set_flags(self, flags: int):
+        """PS_FLAG_* bits; FLAG_FP8 changes the workspace size, so set it before bind()."""
         _check(lib().ps_app_set_flags(self._h, flags), "ps_app_set_flags")
         self.flags = int(flags)
+        self.workspace_bytes = int(lib().ps_app_workspace_bytes(self._h))
 
     def bind(self, inputs, outputs=None, workspace=None, device=None):
         """inputs: per object an f32 CUDA tensor (role in/inout) or None.

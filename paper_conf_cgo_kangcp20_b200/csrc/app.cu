@@ -198,6 +198,11 @@ struct ps_app {
   size_t slot_off[8] = {0};
   size_t partial_off = 0, qparts_off = 0, qres_off = 0, total = 0;
   size_t trans_off[8] = {0};
+  // fp8 (PS_FLAG_FP8, reading #29): per object a staging region of n*8 bytes (the
+  // object decoded into a statement's compute type), its ps_fp8_scale record,
+  // and a vector scratch (MVT's split row-dot)
+  size_t stage_off[8] = {0};
+  size_t scale_off = 0, scratch_off = 0;
   // host-transfer path (ps_run_config_host): per input object, where a2 takes
   // its data from: 0 = orig_in (device conversion), 1 = already in the slot at
   // c(m) (host conversion + H2D), 2 = fp16 intermediate in the transient region
@@ -271,6 +276,18 @@ void layout(ps_app *a) {
   off = align_up(off + (size_t)nout * QBLOCKS_MAX * sizeof(QPart), 256);
   a->qres_off = off;
   off = align_up(off + (size_t)MAX_BATCH * sizeof(QPart), 256);
+  if (a->flags & PS_FLAG_FP8) {
+    size_t vmax = 1;
+    for (int m = 0; m < a->def->nobj; m++) {
+      a->stage_off[m] = off;
+      off = align_up(off + nelem(a, m) * 8, 256);
+      vmax = std::max(vmax, (size_t)std::max(a->rows[m], a->cols[m]));
+    }
+    a->scale_off = off;
+    off = align_up(off + 8 * sizeof(ps_fp8_scale), 256);
+    a->scratch_off = off;
+    off = align_up(off + vmax * 8, 256);
+  }
   for (int m = 0; m < a->def->nobj; m++) {   // transient (fp16 intermediate) region per input
     a->trans_off[m] = off;
     if (a->def->o[m].role == 0 || a->def->o[m].role == 2) off = align_up(off + nelem(a, m) * 2, 256);
@@ -281,7 +298,7 @@ void layout(ps_app *a) {
 // ----------------------------------------------------------- statements
 struct Ctx {
   ps_app *a;
-  const int *prec;
+  int prec[8];      // current storage type of each object (fp8 objects: staged type inside a statement)
   void *ptr[8];
   cudaStream_t st;
   // row-sharded reference: only rows [r0, r1) of the scored output of a
@@ -294,36 +311,110 @@ inline void *eoff(const void *p, int type, int64_t n) {
   return (char *)p + n * (int64_t)dtype_size(type);
 }
 
+// ------------------------------------------------ fp8 staging (reading #29)
+// An fp8 object lives in its slot as codes with a per-tensor scale.  A statement
+// that touches it sees it "staged": decoded into its stage region in the
+// statement's compute type T (exact: RNE_T(q * 2^k)), so every kernel family
+// runs unchanged on f32/f64 storage; objects the statement writes are then
+// re-quantised (amax -> k -> RNE_fp8(v * 2^-k)) back into their slots.  The
+// tcgen05 fp8 contraction reads both multiplicands natively (`native` mask).
+inline unsigned OBJ(int m) { return 1u << m; }
+inline ps_fp8_scale *scale_of(const ps_app *a, int m) {
+  return (ps_fp8_scale *)(a->ws + a->scale_off) + m;
+}
+
+template <class F>
+ps_status stmt(Ctx &c, unsigned reads, unsigned writes, F &&body, unsigned native = 0) {
+  ps_app *a = c.a;
+  const unsigned touched = reads | writes;
+  unsigned f8 = 0;
+  int T = PS_F32;   // R2: widest touched precision, floored at f32 (fp8 codes are narrower)
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!(touched & OBJ(m))) continue;
+    T = widest(T, c.prec[m]);
+    if (is_fp8(c.prec[m]) && !(native & OBJ(m))) f8 |= OBJ(m);
+  }
+  if (!f8) return body();
+  int q[8];
+  void *slot[8];
+  ps_status s;
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!(f8 & OBJ(m))) continue;
+    q[m] = c.prec[m];
+    slot[m] = c.ptr[m];
+    void *stage = a->ws + a->stage_off[m];
+    if (reads & OBJ(m))
+      if ((s = fp8_decode_async(slot[m], q[m], stage, T, nelem(a, m), scale_of(a, m), c.st)) != PS_OK) return s;
+    c.ptr[m] = stage;
+    c.prec[m] = T;
+  }
+  s = body();
+  for (int m = 0; m < a->def->nobj && s == PS_OK; m++) {
+    if (!(f8 & OBJ(m))) continue;
+    if (writes & OBJ(m)) s = fp8_encode_async(c.ptr[m], T, slot[m], q[m], nelem(a, m), scale_of(a, m), c.st);
+    c.ptr[m] = slot[m];
+    c.prec[m] = q[m];
+  }
+  return s;
+}
+
 ps_status contraction(Ctx &c, GemmArgs g) {
-  // tcgen05 for fp16 x fp16 or bf16 x bf16 multiplicands (kind::f16), f32 compute
-  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && g.A.type == g.B.type &&
-                  (g.A.type == PS_F16 || g.A.type == PS_BF16) && g.T == PS_F32 && g.row_off == 0 &&
+  // tcgen05: fp16 x fp16 or bf16 x bf16 (kind::f16), or fp8 x fp8 (kind::f8f6f4,
+  // E4M3/E5M2 in any mix, reading #29); f32 compute
+  const bool pair = (g.A.type == g.B.type && (g.A.type == PS_F16 || g.A.type == PS_BF16)) ||
+                    (is_fp8(g.A.type) && is_fp8(g.B.type));
+  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && pair && g.T == PS_F32 && g.row_off == 0 &&
                   gemm_tc_supported(g);
+  if (!tc && (is_fp8(g.A.type) || is_fp8(g.B.type))) {
+    set_error("internal: fp8 multiplicands reached the SIMT contraction");
+    return PS_ERR_UNSUPPORTED;
+  }
   return tc ? gemm_tc_async(g, c.st) : gemm_simt_async(g, c.st);
+}
+
+// native mask for a contraction X(.)Y -> out: both multiplicands fp8, T = f32 and the
+// tensor-core path takes the shape; otherwise they are staged (SIMT, R3-exact)
+unsigned tc8_native(Ctx &c, int x, int y, std::initializer_list<int> others, GemmArgs g) {
+  if (!is_fp8(c.prec[x]) || !is_fp8(c.prec[y]) || (c.a->flags & PS_FLAG_NO_TENSOR_CORES) || c.sharded())
+    return 0;
+  int T = PS_F32;
+  for (int m : others) T = widest(T, c.prec[m]);
+  if (T != PS_F32) return 0;
+  g.T = PS_F32;
+  g.c_type = PS_F32;                 // the output is staged in f32 when it is fp8
+  if (g.epi == EPI_AXPBY) g.cin_type = PS_F32;
+  return gemm_tc_supported(g) ? (OBJ(x) | OBJ(y)) : 0;
 }
 
 // out(M x N, row-major) = X(M x K, row-major) . Y(K x N, row-major), R3;
 // rows: restrict to the shard's output rows (X and out row-sliced)
-ps_status matmul(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_t K, bool rows = false) {
+GemmArgs matmul_args(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_t K, bool rows) {
   const int64_t r0 = rows && c.sharded() ? c.r0 : 0;
   GemmArgs g{};
   g.M = rows && c.sharded() ? c.r1 - c.r0 : M; g.N = N; g.K = K;
-  g.A = MatDesc{eoff(c.ptr[x], c.prec[x], r0 * K), c.prec[x], K, 1};
-  g.B = MatDesc{c.ptr[y], c.prec[y], N, 1};
+  g.A = MatDesc{eoff(c.ptr[x], c.prec[x], r0 * K), c.prec[x], K, 1, scale_of(c.a, x)};
+  g.B = MatDesc{c.ptr[y], c.prec[y], N, 1, scale_of(c.a, y)};
   g.C = eoff(c.ptr[out], c.prec[out], r0 * N); g.c_type = c.prec[out]; g.ldc = N;
   g.epi = EPI_PLAIN;
   g.T = compute_type({c.prec[x], c.prec[y], c.prec[out]});
-  return g.M > 0 ? contraction(c, g) : PS_OK;
+  return g;
+}
+ps_status matmul(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_t K, bool rows = false) {
+  const unsigned nat = tc8_native(c, x, y, {out}, matmul_args(c, x, y, out, M, N, K, rows));
+  return stmt(c, OBJ(x) | OBJ(y), OBJ(out), [&]() -> ps_status {
+    GemmArgs g = matmul_args(c, x, y, out, M, N, K, rows);
+    return g.M > 0 ? contraction(c, g) : PS_OK;
+  }, nat);
 }
 
 // symmat(M x M) = data^T data over N rows, upper tiles + mirror (R3).  Sharded: the
 // upper part of rows [r0, r1) only; the mirror runs after the gather (reference_merge)
-ps_status syrk(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double div, int diag_one) {
+GemmArgs syrk_args(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double div) {
   const int64_t r0 = c.sharded() ? c.r0 : 0;
   GemmArgs g{};
   g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
-  g.A = MatDesc{eoff(c.ptr[data], c.prec[data], r0), c.prec[data], 1, M};   // A(j1, i) = data[i][j1]
-  g.B = MatDesc{c.ptr[data], c.prec[data], M, 1};                          // B(i, j2) = data[i][j2]
+  g.A = MatDesc{eoff(c.ptr[data], c.prec[data], r0), c.prec[data], 1, M, scale_of(c.a, data)};   // A(j1, i) = data[i][j1]
+  g.B = MatDesc{c.ptr[data], c.prec[data], M, 1, scale_of(c.a, data)};                          // B(i, j2) = data[i][j2]
   g.C = eoff(c.ptr[sym], c.prec[sym], r0 * M); g.c_type = c.prec[sym]; g.ldc = M;
   g.epi = epi; g.div = div;
   if (epi == EPI_AXPBY) {   // SYRK app: C <- alpha data^T data + beta C (C read in place)
@@ -333,16 +424,58 @@ ps_status syrk(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double 
   g.upper_only = 1;
   g.row_off = r0;
   g.T = compute_type({c.prec[data], c.prec[sym]});
-  if (g.M <= 0) return PS_OK;
-  ps_status s = contraction(c, g);
-  if (s != PS_OK || c.sharded()) return s;
-  return mirror_async(c.ptr[sym], c.prec[sym], M, diag_one, c.st);
+  return g;
+}
+ps_status syrk(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, double div, int diag_one) {
+  const unsigned nat = tc8_native(c, data, data, {sym}, syrk_args(c, data, sym, N, M, epi, div));
+  const unsigned reads = OBJ(data) | (epi == EPI_AXPBY ? OBJ(sym) : 0u);
+  return stmt(c, reads, OBJ(sym), [&]() -> ps_status {
+    GemmArgs g = syrk_args(c, data, sym, N, M, epi, div);
+    if (g.M <= 0) return PS_OK;
+    ps_status s = contraction(c, g);
+    if (s != PS_OK || c.sharded()) return s;
+    return mirror_async(c.ptr[sym], c.prec[sym], M, diag_one, c.st);
+  }, nat);
+}
+
+GemmArgs gemm_args(Ctx &c) {   // C <- alpha (A.B) + beta C
+  const int64_t *d = c.a->d;
+  const int64_t r0 = c.sharded() ? c.r0 : 0;
+  GemmArgs g{};
+  g.M = c.sharded() ? c.r1 - c.r0 : d[0]; g.N = d[1]; g.K = d[2];
+  g.A = MatDesc{eoff(c.ptr[0], c.prec[0], r0 * d[2]), c.prec[0], d[2], 1, scale_of(c.a, 0)};
+  g.B = MatDesc{c.ptr[1], c.prec[1], d[1], 1, scale_of(c.a, 1)};
+  g.C = eoff(c.ptr[2], c.prec[2], r0 * d[1]); g.c_type = c.prec[2]; g.ldc = d[1];
+  g.Cin = g.C; g.cin_type = c.prec[2];
+  g.epi = EPI_AXPBY; g.alpha = c.a->sc[0]; g.beta = c.a->sc[1];
+  g.T = compute_type({c.prec[0], c.prec[1], c.prec[2]});
+  return g;
+}
+
+GemmArgs syr2k_args(Ctx &c, int s2) {   // C <- alpha X^T Y + beta C (s2 = 0: X=A, Y=B; 1: X=B, Y=A, beta 1)
+  const int64_t N = c.a->d[0], M = c.a->d[1], r0 = c.sharded() ? c.r0 : 0;
+  const int x = s2 ? 1 : 0, y = s2 ? 0 : 1;
+  GemmArgs g{};
+  g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
+  g.A = MatDesc{eoff(c.ptr[x], c.prec[x], r0), c.prec[x], 1, M, scale_of(c.a, x)};   // A(i, k) = X[k][i]
+  g.B = MatDesc{c.ptr[y], c.prec[y], M, 1, scale_of(c.a, y)};                       // B(k, j) = Y[k][j]
+  g.C = eoff(c.ptr[2], c.prec[2], r0 * M); g.c_type = c.prec[2]; g.ldc = M;
+  g.Cin = g.C; g.cin_type = c.prec[2];
+  g.epi = EPI_AXPBY; g.alpha = c.a->sc[0]; g.beta = s2 ? 1.0 : c.a->sc[1];
+  g.T = compute_type({c.prec[0], c.prec[1], c.prec[2]});
+  return g;
+}
+
+bool any_fp8(const Ctx &c, unsigned mask) {
+  for (int m = 0; m < c.a->def->nobj; m++)
+    if ((mask & OBJ(m)) && is_fp8(c.prec[m])) return true;
+  return false;
 }
 
 ps_status run_statements(Ctx &c) {
   ps_app *a = c.a;
   const int64_t *d = a->d;
-  const int *p = c.prec;
+  const int *p = c.prec;     // current storage types (staged inside stmt bodies)
   void **P = c.ptr;
   void *partial = a->ws + a->partial_off;
   ps_status s = PS_OK;
@@ -352,16 +485,11 @@ ps_status run_statements(Ctx &c) {
   } while (0)
   switch (a->kind) {
     case K_GEMM: {   // C <- alpha (A.B) + beta C
-      const int64_t r0 = c.sharded() ? c.r0 : 0;
-      GemmArgs g{};
-      g.M = c.sharded() ? c.r1 - c.r0 : d[0]; g.N = d[1]; g.K = d[2];
-      g.A = MatDesc{eoff(P[0], p[0], r0 * d[2]), p[0], d[2], 1};
-      g.B = MatDesc{P[1], p[1], d[1], 1};
-      g.C = eoff(P[2], p[2], r0 * d[1]); g.c_type = p[2]; g.ldc = d[1];
-      g.Cin = g.C; g.cin_type = p[2];
-      g.epi = EPI_AXPBY; g.alpha = a->sc[0]; g.beta = a->sc[1];
-      g.T = compute_type({p[0], p[1], p[2]});
-      if (g.M > 0) S_(contraction(c, g));
+      const unsigned nat = tc8_native(c, 0, 1, {2}, gemm_args(c));
+      S_(stmt(c, OBJ(0) | OBJ(1) | OBJ(2), OBJ(2), [&]() -> ps_status {
+        GemmArgs g = gemm_args(c);
+        return g.M > 0 ? contraction(c, g) : PS_OK;
+      }, nat));
       break;
     }
     case K_2MM:
@@ -374,77 +502,135 @@ ps_status run_statements(Ctx &c) {
       S_(matmul(c, 4, 5, 6, d[0], d[3], d[1], true));   // G <- E.F
       break;
     case K_ATAX:   // tmp <- A x ; y <- A^T tmp
-      S_(rowdot_async(P[0], p[0], d[1], P[1], p[1], P[3], p[3], d[0], d[1], partial, c.st));
-      S_(colsum_async(P[0], p[0], d[1], P[3], p[3], P[2], p[2], d[0], d[1],
-                      compute_type({p[0], p[3], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st));
+      S_(stmt(c, OBJ(0) | OBJ(1), OBJ(3), [&] {
+        return rowdot_async(P[0], p[0], d[1], P[1], p[1], P[3], p[3], d[0], d[1], partial, c.st);
+      }));
+      S_(stmt(c, OBJ(0) | OBJ(3), OBJ(2), [&] {
+        return colsum_async(P[0], p[0], d[1], P[3], p[3], P[2], p[2], d[0], d[1],
+                            compute_type({p[0], p[3], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st);
+      }));
       break;
     case K_BICG:   // s <- A^T r ; q <- A p   (one pass over A)
-      S_(bicg_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], P[3], p[3], P[4], p[4], d[0], d[1],
-                    partial, c.st));
+      if (!any_fp8(c, 0x1Fu)) {
+        S_(bicg_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], P[3], p[3], P[4], p[4], d[0], d[1],
+                      partial, c.st));
+      } else {   // fp8 objects: the two statements separately (each stages A in its own T)
+        S_(stmt(c, OBJ(0) | OBJ(1), OBJ(2), [&] {
+          return colsum_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], d[0], d[1],
+                              compute_type({p[0], p[1], p[2]}), COL_DOT, FIN_PLAIN, 0, 0, partial, c.st);
+        }));
+        S_(stmt(c, OBJ(0) | OBJ(3), OBJ(4), [&] {
+          return rowdot_async(P[0], p[0], d[1], P[3], p[3], P[4], p[4], d[0], d[1], partial, c.st);
+        }));
+      }
       break;
     case K_GESUMMV:   // tmp <- A x ; y <- B x ; y <- alpha tmp + beta y
-      S_(rowdot_async(P[0], p[0], d[0], P[2], p[2], P[4], p[4], d[0], d[0], partial, c.st));
-      S_(rowdot_async(P[1], p[1], d[0], P[2], p[2], P[3], p[3], d[0], d[0], partial, c.st));
-      S_(axpby_async(P[4], p[4], P[3], p[3], d[0], a->sc[0], a->sc[1], c.st));
+      S_(stmt(c, OBJ(0) | OBJ(2), OBJ(4), [&] {
+        return rowdot_async(P[0], p[0], d[0], P[2], p[2], P[4], p[4], d[0], d[0], partial, c.st);
+      }));
+      S_(stmt(c, OBJ(1) | OBJ(2), OBJ(3), [&] {
+        return rowdot_async(P[1], p[1], d[0], P[2], p[2], P[3], p[3], d[0], d[0], partial, c.st);
+      }));
+      S_(stmt(c, OBJ(4) | OBJ(3), OBJ(3), [&] {
+        return axpby_async(P[4], p[4], P[3], p[3], d[0], a->sc[0], a->sc[1], c.st);
+      }));
       break;
     case K_CORR: {
       const double n = (double)d[0];
-      S_(colsum_async(P[0], p[0], d[1], nullptr, PS_F32, P[1], p[1], d[0], d[1],
-                      compute_type({p[0], p[1]}), COL_SUM, FIN_MEAN, n, 0, partial, c.st));
-      S_(colsum_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], d[0], d[1],
-                      compute_type({p[0], p[1], p[2]}), COL_SQDEV, FIN_STDDEV, n, a->sc[0],
-                      partial, c.st));
-      S_(corr_normalize_async(P[0], p[0], P[1], p[1], P[2], p[2], d[0], d[1], sqrt(n), c.st));
+      S_(stmt(c, OBJ(0), OBJ(1), [&] {
+        return colsum_async(P[0], p[0], d[1], nullptr, PS_F32, P[1], p[1], d[0], d[1],
+                            compute_type({p[0], p[1]}), COL_SUM, FIN_MEAN, n, 0, partial, c.st);
+      }));
+      S_(stmt(c, OBJ(0) | OBJ(1), OBJ(2), [&] {
+        return colsum_async(P[0], p[0], d[1], P[1], p[1], P[2], p[2], d[0], d[1],
+                            compute_type({p[0], p[1], p[2]}), COL_SQDEV, FIN_STDDEV, n, a->sc[0],
+                            partial, c.st);
+      }));
+      S_(stmt(c, OBJ(0) | OBJ(1) | OBJ(2), OBJ(0), [&] {
+        return corr_normalize_async(P[0], p[0], P[1], p[1], P[2], p[2], d[0], d[1], sqrt(n), c.st);
+      }));
       S_(syrk(c, 0, 3, d[0], d[1], EPI_PLAIN, 0.0, 1));
       break;
     }
     case K_COVAR: {
       const double n = (double)d[0];
-      S_(colsum_async(P[0], p[0], d[1], nullptr, PS_F32, P[1], p[1], d[0], d[1],
-                      compute_type({p[0], p[1]}), COL_SUM, FIN_MEAN, n, 0, partial, c.st));
-      S_(covar_center_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st));
+      S_(stmt(c, OBJ(0), OBJ(1), [&] {
+        return colsum_async(P[0], p[0], d[1], nullptr, PS_F32, P[1], p[1], d[0], d[1],
+                            compute_type({p[0], p[1]}), COL_SUM, FIN_MEAN, n, 0, partial, c.st);
+      }));
+      S_(stmt(c, OBJ(0) | OBJ(1), OBJ(0), [&] {
+        return covar_center_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st);
+      }));
       S_(syrk(c, 0, 2, d[0], d[1], EPI_DIV, n - 1.0, 0));
       break;
     }
     case K_MVT:   // x1 <- x1 + A y1 ; x2 <- x2 + A^T y2   (one pass over A)
-      S_(mvt_async(P[0], p[0], d[0], P[1], p[1], P[2], p[2], P[3], p[3], P[4], p[4], partial, c.st));
+      if (!any_fp8(c, 0x1Fu)) {
+        S_(mvt_async(P[0], p[0], d[0], P[1], p[1], P[2], p[2], P[3], p[3], P[4], p[4], partial, c.st));
+      } else {   // fp8 objects: row-dot into a T-typed scratch, x1 = fma(1, dot, 1 * x1); colsum + add
+        void *scratch = a->ws + a->scratch_off;
+        S_(stmt(c, OBJ(0) | OBJ(1) | OBJ(3), OBJ(1), [&] {
+          const int T1 = compute_type({p[0], p[1], p[3]});
+          ps_status e = rowdot_async(P[0], p[0], d[0], P[3], p[3], scratch, T1, d[0], d[0], partial, c.st);
+          return e != PS_OK ? e : axpby_async(scratch, T1, P[1], p[1], d[0], 1.0, 1.0, c.st);
+        }));
+        S_(stmt(c, OBJ(0) | OBJ(2) | OBJ(4), OBJ(2), [&] {
+          return colsum_async(P[0], p[0], d[0], P[4], p[4], P[2], p[2], d[0], d[0],
+                              compute_type({p[0], p[2], p[4]}), COL_DOT, FIN_ADD, 0, 0, partial, c.st);
+        }));
+      }
       break;
     case K_SYRK:  // C <- alpha A^T A + beta C (upper tiles, mirrored)
       S_(syrk(c, 0, 1, d[0], d[1], EPI_AXPBY, 0.0, 0));
       break;
     case K_CONV2D:
-      S_(conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st));
+      S_(stmt(c, OBJ(0), OBJ(1), [&] { return conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st); }));
       break;
     case K_SYR2K: {   // C <- alpha A^T B + beta C ; C <- alpha B^T A + C
-      const int64_t N = d[0], M = d[1], r0 = c.sharded() ? c.r0 : 0;
       for (int s2 = 0; s2 < 2; s2++) {
-        const int x = s2 ? 1 : 0, y = s2 ? 0 : 1;
-        GemmArgs g{};
-        g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
-        g.A = MatDesc{eoff(P[x], p[x], r0), p[x], 1, M};   // A(i, k) = X[k][i]
-        g.B = MatDesc{P[y], p[y], M, 1};                   // B(k, j) = Y[k][j]
-        g.C = eoff(P[2], p[2], r0 * M); g.c_type = p[2]; g.ldc = M;
-        g.Cin = g.C; g.cin_type = p[2];
-        g.epi = EPI_AXPBY; g.alpha = a->sc[0]; g.beta = s2 ? 1.0 : a->sc[1];
-        g.T = compute_type({p[0], p[1], p[2]});
-        if (g.M > 0) S_(contraction(c, g));
+        const unsigned nat = tc8_native(c, 0, 1, {2}, syr2k_args(c, s2));
+        S_(stmt(c, OBJ(0) | OBJ(1) | OBJ(2), OBJ(2), [&]() -> ps_status {
+          GemmArgs g = syr2k_args(c, s2);
+          return g.M > 0 ? contraction(c, g) : PS_OK;
+        }, nat));
       }
       break;
     }
     case K_CONV3D:
-      S_(conv3d_async(P[0], p[0], P[1], p[1], d[0], d[1], d[2], c.st));
+      S_(stmt(c, OBJ(0), OBJ(1), [&] { return conv3d_async(P[0], p[0], P[1], p[1], d[0], d[1], d[2], c.st); }));
       break;
-    case K_FDTD2D:
-      for (int64_t t = 0; t < d[0]; t++)
-        S_(fdtd2d_step_async(P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st));
+    case K_FDTD2D: {
+      // statements per step (reading #27); with fp8 objects the ey row-0 assignment and
+      // the ey update are separate statements (reading #29), otherwise one fused pass
+      const bool f8 = any_fp8(c, 0xFu);
+      for (int64_t t = 0; t < d[0]; t++) {
+        if (!f8) {
+          S_(fdtd2d_part_async(FDTD_EY, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st));
+        } else {
+          S_(stmt(c, OBJ(0) | OBJ(2), OBJ(2), [&] {
+            return fdtd2d_part_async(FDTD_EY0, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st);
+          }));
+          S_(stmt(c, OBJ(2) | OBJ(3), OBJ(2), [&] {
+            return fdtd2d_part_async(FDTD_EY1, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st);
+          }));
+        }
+        S_(stmt(c, OBJ(1) | OBJ(3), OBJ(1), [&] {
+          return fdtd2d_part_async(FDTD_EX, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st);
+        }));
+        S_(stmt(c, OBJ(1) | OBJ(2) | OBJ(3), OBJ(3), [&] {
+          return fdtd2d_part_async(FDTD_HZ, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], d[2], c.st);
+        }));
+      }
       break;
+    }
   }
 #undef S_
   return PS_OK;
 }
 
-// configuration alphabet: the paper's {f64, f32, f16}, or + bf16 (PS_FLAG_BF16, reading #28)
-int radix(const ps_app *a) { return (a->flags & PS_FLAG_BF16) ? 4 : 3; }
+// configuration alphabet: the paper's {f64, f32, f16}, + bf16 (PS_FLAG_BF16, reading #28),
+// + bf16, e4m3, e5m2 (PS_FLAG_FP8, reading #29)
+int radix(const ps_app *a) { return (a->flags & PS_FLAG_FP8) ? 6 : ((a->flags & PS_FLAG_BF16) ? 4 : 3); }
 
 ps_status check_prec(const ps_app *a, const int *prec) {
   if (!prec) { set_error("null precision vector"); return PS_ERR_INVALID; }
@@ -477,7 +663,8 @@ ps_status ensure_events(ps_app *a, size_t n) {
 // rows [r0, r1) of the scored output (row-sharded reference, no quality)
 ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res,
                          cudaEvent_t *ev, bool quality, int64_t r0 = 0, int64_t r1 = -1) {
-  Ctx c{a, prec, {nullptr}, st};
+  Ctx c{a, {0}, {nullptr}, st};
+  for (int m = 0; m < a->def->nobj; m++) c.prec[m] = prec[m];
   c.r0 = r0;
   c.r1 = r1;
   if (ev) PS_CUDA(cudaEventRecord(ev[0], st));
@@ -492,6 +679,9 @@ ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res
         if (s != PS_OK) return s;
       } else if (role == 0 && prec[m] == PS_F32) {
         c.ptr[m] = (void *)a->orig_in[m];   // original precision: used in place
+      } else if (is_fp8(prec[m])) {         // reading #29: amax -> k -> codes
+        ps_status s = fp8_encode_async(a->orig_in[m], PS_F32, c.ptr[m], prec[m], nelem(a, m), scale_of(a, m), st);
+        if (s != PS_OK) return s;
       } else {
         ps_status s = convert_async(a->orig_in[m], PS_F32, c.ptr[m], prec[m], nelem(a, m), st);
         if (s != PS_OK) return s;
@@ -507,8 +697,16 @@ ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res
   int np = 0;
   for (int m = 0; m < a->def->nobj; m++) {
     if (!a->def->o[m].is_output) continue;
-    s = backconv_quality_async(c.ptr[m], prec[m], a->ref[m], a->orig_out[m], nelem(a, m),
-                               parts + np, st);
+    const void *out = c.ptr[m];
+    int ot = prec[m];
+    if (is_fp8(ot)) {   // reading #29: the exact values q * 2^k, then as an f64 object
+      void *stage = a->ws + a->stage_off[m];
+      s = fp8_decode_async(out, ot, stage, PS_F64, nelem(a, m), scale_of(a, m), st);
+      if (s != PS_OK) return s;
+      out = stage;
+      ot = PS_F64;
+    }
+    s = backconv_quality_async(out, ot, a->ref[m], a->orig_out[m], nelem(a, m), parts + np, st);
     if (s != PS_OK) return s;
     np += qblocks(nelem(a, m));
   }
@@ -649,7 +847,12 @@ ps_status ps_app_object_info(const ps_app *a, int m, ps_object_info *out) {
 
 ps_status ps_app_set_flags(ps_app *a, uint32_t flags) {
   if (!a) { set_error("null app"); return PS_ERR_INVALID; }
+  if (a->bound && ((flags ^ a->flags) & PS_FLAG_FP8)) {
+    set_error("ps_app_set_flags: PS_FLAG_FP8 changes the workspace layout; set it before ps_app_bind");
+    return PS_ERR_INVALID;
+  }
   a->flags = flags;
+  layout(a);
   return PS_OK;
 }
 
@@ -853,7 +1056,10 @@ ps_status ps_sweep(ps_app *a, const uint64_t *ids, size_t n, double toq, void *s
 }
 
 ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, int threads, int simd) {
-  if (!dtype_ok(dst_type)) { set_error("ps_host_convert: bad dtype"); return PS_ERR_INVALID; }
+  if (!dtype_ok(dst_type) || is_fp8(dst_type)) {   // fp8: the scale needs a device amax pass
+    set_error("ps_host_convert: bad dtype (fp8 objects convert on the device)");
+    return PS_ERR_INVALID;
+  }
   if (n && (!src || !dst)) { set_error("ps_host_convert: null pointer"); return PS_ERR_INVALID; }
   ps::host_convert_f32(src, dst, dst_type, n, threads, simd != 0);
   return PS_OK;
@@ -863,7 +1069,7 @@ ps_status ps_host_convert(const float *src, void *dst, int dst_type, size_t n, i
 static thread_local XferScratch g_xs;
 ps_status ps_transfer(const float *host_src, void *dev_dst, int dst_type, size_t n, int method,
                       int threads, void *dev_stage, void *stream, float *ms) {
-  if (!dtype_ok(dst_type) || method < PS_XFER_DEVICE || method > PS_XFER_TRANSIENT) {
+  if (!dtype_ok(dst_type) || is_fp8(dst_type) || method < PS_XFER_DEVICE || method > PS_XFER_TRANSIENT) {
     set_error("ps_transfer: bad dtype or method");
     return PS_ERR_INVALID;
   }
@@ -916,8 +1122,10 @@ ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
     a->pre[m] = 0;
     if (role != 0 && role != 2) continue;
     int meth = methods ? methods[m] : PS_XFER_DEVICE;
-    // an f32 input already has its precision: H2D at orig, used in place by a2
+    // an f32 input already has its precision: H2D at orig, used in place by a2; an fp8
+    // object's scale needs its amax on the device (reading #29): device method
     if (prec[m] == PS_F32 && role == 0 && meth != PS_XFER_TRANSIENT) meth = PS_XFER_DEVICE;
+    if (is_fp8(prec[m])) meth = PS_XFER_DEVICE;
     void *stage = meth == PS_XFER_TRANSIENT ? (void *)(a->ws + a->trans_off[m]) : (void *)a->orig_in[m];
     s = xfer_object(a->xs, (const float *)host_inputs[m], nelem(a, m), prec[m], meth, threads,
                     a->ws + a->slot_off[m], stage, st);

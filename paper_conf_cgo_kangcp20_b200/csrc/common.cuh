@@ -34,8 +34,9 @@ void count_launch();
     if (_e != cudaSuccess) return ps::cuda_status(_e, what);  \
   } while (0)
 
-inline size_t dtype_size(int t) { return t == PS_F64 ? 8 : (t == PS_F32 ? 4 : 2); }
-inline bool dtype_ok(int t) { return t == PS_F64 || t == PS_F32 || t == PS_F16 || t == PS_BF16; }
+inline bool is_fp8(int t) { return t == PS_E4M3 || t == PS_E5M2; }
+inline size_t dtype_size(int t) { return t == PS_F64 ? 8 : (t == PS_F32 ? 4 : (is_fp8(t) ? 1 : 2)); }
+inline bool dtype_ok(int t) { return t >= PS_F64 && t <= PS_E5M2; }
 // R2: compute type = widest (smallest code) floored at f32
 inline int widest(int a, int b) { return a < b ? a : b; }
 inline int compute_type(std::initializer_list<int> ts) {
@@ -48,12 +49,16 @@ int num_sms();
 // ------------------------------------------------------- storage traits
 struct F16 { uint16_t b; };    // tag type for fp16 storage (IEEE binary16 bits)
 struct BF16 { uint16_t b; };   // tag type for bf16 storage (reading #28)
+struct E4M3 { uint8_t b; };    // fp8 storage tags (reading #29): raw codes, the
+struct E5M2 { uint8_t b; };    // per-tensor scale lives beside the object
 
 template <class S> struct Store;
 template <> struct Store<double> { using raw = double; static constexpr int code = PS_F64; };
 template <> struct Store<float> { using raw = float; static constexpr int code = PS_F32; };
 template <> struct Store<F16> { using raw = uint16_t; static constexpr int code = PS_F16; };
 template <> struct Store<BF16> { using raw = uint16_t; static constexpr int code = PS_BF16; };
+template <> struct Store<E4M3> { using raw = uint8_t; static constexpr int code = PS_E4M3; };
+template <> struct Store<E5M2> { using raw = uint8_t; static constexpr int code = PS_E5M2; };
 
 // exact widening of a stored element to T (NaN payloads are irrelevant for
 // arithmetic: any NaN propagates and is scored as non-finite)
@@ -145,6 +150,43 @@ template <class T> struct St<F16, T> {
 template <class T> struct St<BF16, T> {
   static __device__ __forceinline__ void put(uint16_t *p, size_t i, T v) { p[i] = rne_bf16(v); }
 };
+
+// ------------------------------------------------ fp8 codes (reading #29)
+// E4M3 (OCP "fn": no inf, NaN 0x7F/0xFF, max 448) and E5M2 (IEEE-like, max 57344).
+// Decoding a code is exact in f16 (and therefore in f32 / f64).
+__device__ __forceinline__ float fp8_to_f32(uint8_t q, bool e4m3) {
+  uint32_t h2;
+  const uint16_t in = q;
+  if (e4m3) asm("cvt.rn.f16x2.e4m3x2 %0, %1;" : "=r"(h2) : "h"(in));
+  else asm("cvt.rn.f16x2.e5m2x2 %0, %1;" : "=r"(h2) : "h"(in));
+  return f16_to_f32((uint16_t)(h2 & 0xFFFFu));
+}
+// RNE of a finite-or-not f32 y to the fp8 code: non-finite inputs and
+// magnitudes past the overflow midpoint follow the oracle (E4M3: NaN 0x7F; E5M2:
+// +-inf), NaN -> canonical 0x7F; the satfinite cvt is only reached in range.
+__device__ __forceinline__ uint8_t f32_to_fp8(float y, bool e4m3) {
+  const uint32_t sign = (__float_as_uint(y) >> 24) & 0x80u;
+  const float a = fabsf(y);
+  if (y != y) return 0x7F;
+  if (e4m3) {
+    if (a > 464.0f) return 0x7F;                    // 464 is the 448/480 tie -> 448
+  } else {
+    if (a >= 61440.0f) return (uint8_t)(sign | 0x7Cu);   // 61440: 57344/65536 tie -> inf
+  }
+  uint16_t r;
+  if (e4m3) asm("cvt.rn.satfinite.e4m3x2.f32 %0, %1, %2;" : "=h"(r) : "f"(0.0f), "f"(y));
+  else asm("cvt.rn.satfinite.e5m2x2.f32 %0, %1, %2;" : "=h"(r) : "f"(0.0f), "f"(y));
+  return (uint8_t)(r & 0xFFu);
+}
+// f64 -> fp8 in ONE rounding: round-to-odd to f32 (24 bits >= 4 + 2), then RNE
+__device__ __forceinline__ uint8_t f64_to_fp8(double x, bool e4m3) {
+  if (x != x) return 0x7F;
+  float f;
+  asm("cvt.rz.f32.f64 %0, %1;" : "=f"(f) : "d"(x));
+  if ((double)f != x && !isinf(x)) f = __uint_as_float(__float_as_uint(f) | 1u);
+  if (isinf(x)) f = (float)x;
+  return f32_to_fp8(f, e4m3);
+}
 
 // R4 arithmetic helpers (explicit FMA; everything else is plain IEEE)
 __device__ __forceinline__ float t_fma(float a, float b, float c) { return __fmaf_rn(a, b, c); }

@@ -14,6 +14,7 @@
 #include <cstring>
 
 #include "common.cuh"
+#include "kernels.cuh"
 
 namespace ps {
 
@@ -168,6 +169,12 @@ ps_status convert_async(const void *src, int st, void *dst, int dt, size_t n, cu
     PS_CUDA(cudaMemcpyAsync(dst, src, n * dtype_size(st), cudaMemcpyDeviceToDevice, stream));
     return PS_OK;
   }
+  if (is_fp8(st) && is_fp8(dt)) {
+    set_error("ps_convert: e4m3 <-> e5m2 is not supported");
+    return PS_ERR_UNSUPPORTED;
+  }
+  if (is_fp8(dt)) return fp8_encode_async(src, st, dst, dt, n, nullptr, stream);   // unscaled
+  if (is_fp8(st)) return fp8_decode_async(src, st, dst, dt, n, nullptr, stream);
   if (st == PS_F32 && dt == PS_F16) return launch_convert<float, F16>(src, dst, n, stream);
   if (st == PS_F64 && dt == PS_F16) return launch_convert<double, F16>(src, dst, n, stream);
   if (st == PS_F64 && dt == PS_F32) return launch_convert<double, float>(src, dst, n, stream);

@@ -17,6 +17,12 @@
 //                      32*(w%4)..), alpha/beta or divide in f32, RNE store to
 //                      the output object's precision (R1)
 // A may be K-major (row-major A) or M-major (SYRK's data^T); B is N-major.
+//
+// fp8 x fp8 (reading #29; kind::f8f6f4, E4M3/E5M2 in any mix): the same
+// kernels instantiated with 1-byte elements -- a k-block is 128 elements (still
+// one 128-byte swizzled row), each MMA consumes K = 32, MN-major boxes are 128
+// elements wide; the epilogue multiplies the f32 accumulator by the operands'
+// per-tensor scales 2^(ka + kb) (exact) before alpha/beta.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -26,14 +32,22 @@
 namespace ps {
 namespace tc {
 
-constexpr int BM = 128, BN = 256, BK = 64, STAGES = 4;
-constexpr int A_BYTES = BM * BK * 2;            // 16 KiB
-constexpr int B_BYTES = BN * BK * 2;            // 32 KiB
+constexpr int BM = 128, BN = 256, STAGES = 4;
+constexpr int KB_BYTES = 128;                   // one k-block = one 128-byte swizzled row
+constexpr int A_BYTES = BM * KB_BYTES;          // 16 KiB
+constexpr int B_BYTES = BN * KB_BYTES;          // 32 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
 constexpr int NTHREADS = 192;
 constexpr uint32_t TMEM_COLS = 256;
-constexpr uint32_t BOX_BYTES = 64 * 64 * 2;    // one 64 (MN) x 64 (K) box = 8 KiB
+// element-size dependent geometry (ES = 2: f16/bf16, ES = 1: fp8)
+template <int ES> struct Geo {
+  static constexpr int BK = KB_BYTES / ES;              // elements per k-block
+  static constexpr int MN_BOX = 128 / ES;               // MN-major box width (elements)
+  static constexpr uint32_t BOX_BYTES = 128 * BK;       // one MN-major box {MN_BOX, BK}
+  static constexpr int MMA_K = 32 / ES;                 // K per tcgen05.mma
+  static constexpr uint32_t MN_STEP = MMA_K * 128;      // MN-major: bytes per MMA k-step
+};
 
 struct Params {
   int M, N, K;
@@ -46,7 +60,8 @@ struct Params {
   int epi;
   float alpha, beta, div;
   int upper_only;
-  uint32_t ab_fmt;   // kind::f16 operand format: 0 = f16, 1 = bf16 (reading #28)
+  uint32_t a_fmt, b_fmt;   // kind::f16: 0 = f16, 1 = bf16 (reading #28); kind::f8f6f4: 0 = E4M3, 1 = E5M2
+  const ps_fp8_scale *sa, *sb;   // fp8 operands: per-tensor scales (reading #29)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -93,13 +108,25 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
   d |= (uint64_t)2 << 61;
   return d;
 }
+template <int ES>
 __device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc,
                                          uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(a), "l"(b), "r"(idesc), "r"(accumulate));
+  if constexpr (ES == 2)
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(idesc), "r"(accumulate));
+  else
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f8f6f4 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(idesc), "r"(accumulate));
+}
+// the fp8 operands' scale 2^(ka + kb); 1 for f16 / bf16
+__device__ __forceinline__ int scale_exp2(const Params &p) {
+  return (p.sa ? p.sa->k : 0) + (p.sb ? p.sb->k : 0);
 }
 __device__ __forceinline__ void umma_commit(uint64_t *bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
@@ -134,9 +161,12 @@ __device__ __forceinline__ void store_c(void *p, int type, int64_t idx, float v)
   else ((uint16_t *)p)[idx] = rne_f16(v);
 }
 
+template <int ES>
 __global__ void __launch_bounds__(NTHREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
                    Params p) {
+  using G = Geo<ES>;
+  constexpr int BK = G::BK;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t *sA = smem;
@@ -182,20 +212,22 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const int k0 = kb * BK;
         uint8_t *a = sA + s * A_BYTES;
         if (!p.a_mn_major) {
-          tma_load_2d(a, &tma_a, &full[s], k0, m0);                 // box {64 K, 128 M}
+          tma_load_2d(a, &tma_a, &full[s], k0, m0);                 // box {BK, 128 M}
         } else {
-          tma_load_2d(a, &tma_a, &full[s], m0, k0);                 // box {64 M, 64 K} x 2
-          tma_load_2d(a + BOX_BYTES, &tma_a, &full[s], m0 + 64, k0);
+#pragma unroll
+          for (int q = 0; q < BM / G::MN_BOX; q++)                  // box {MN_BOX M, BK}
+            tma_load_2d(a + q * G::BOX_BYTES, &tma_a, &full[s], m0 + G::MN_BOX * q, k0);
         }
         uint8_t *b = sB + s * B_BYTES;
 #pragma unroll
-        for (int q = 0; q < BN / 64; q++) tma_load_2d(b + q * BOX_BYTES, &tma_b, &full[s], n0 + 64 * q, k0);
+        for (int q = 0; q < BN / G::MN_BOX; q++)
+          tma_load_2d(b + q * G::BOX_BYTES, &tma_b, &full[s], n0 + G::MN_BOX * q, k0);
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {   // ---------------- MMA issuer (single thread)
       const uint32_t idesc = (1u << 4)                          // D = f32
-                             | (p.ab_fmt << 7) | (p.ab_fmt << 10)   // A, B format
+                             | (p.a_fmt << 7) | (p.b_fmt << 10)     // A, B format
                              | ((uint32_t)p.a_mn_major << 15)   // A major
                              | (1u << 16)                       // B is N-major
                              | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
@@ -206,13 +238,13 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         fence_after();
         const uint32_t abase = smem_u32(sA + s * A_BYTES), bbase = smem_u32(sB + s * B_BYTES);
 #pragma unroll
-        for (int kk = 0; kk < BK / 16; kk++) {
-          // K-major SW128: +32 B per 16-element K step inside the 128 B swizzled row;
-          // MN-major SW128: +2 KiB (16 K-rows of 128 B); LBO = 8 KiB between 64-wide boxes.
-          const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * 2048, BOX_BYTES, 1024)
+        for (int kk = 0; kk < BK / G::MMA_K; kk++) {
+          // K-major SW128: +32 B per MMA K step inside the 128 B swizzled row;
+          // MN-major SW128: +MMA_K K-rows of 128 B; LBO = one MN box between boxes.
+          const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * G::MN_STEP, G::BOX_BYTES, 1024)
                                            : umma_desc(abase + kk * 32, 16, 1024);
-          const uint64_t bd = umma_desc(bbase + kk * 2048, BOX_BYTES, 1024);
-          umma_f16(tmem, ad, bd, idesc, (kb | kk) != 0);
+          const uint64_t bd = umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
+          umma_f16<ES>(tmem, ad, bd, idesc, (kb | kk) != 0);
         }
         umma_commit(&empty[s]);   // frees the stage when these MMAs retire
       }
@@ -221,6 +253,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   } else {   // ------------------------- epilogue warps 2..5
     mbar_wait(tfull, 0);
     fence_after();
+    const int kab = scale_exp2(p);
     const int q = warp & 3;                 // TMEM lane quarter this warp may access
     const int64_t row = (int64_t)m0 + q * 32 + lane;
     for (int cc = 0; cc < BN / 16; cc++) {
@@ -232,6 +265,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const int64_t col = (int64_t)n0 + cc * 16 + e;
           if (col >= p.N) break;
           float r = __uint_as_float(v[e]);
+          if (ES == 1) r = scalbnf(r, kab);   // exact power-of-two scale
           const int64_t idx = row * p.ldc + col;
           if (p.epi == EPI_AXPBY) r = __fmaf_rn(p.alpha, r, p.beta * load_c(p.Cin, p.cin_type, idx));
           else if (p.epi == EPI_DIV) r = r / p.div;
@@ -259,10 +293,10 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 // c, c + #clusters, ... (SYRK: lower tiles skipped by every role alike).
 namespace tc2 {
 
-constexpr int BM = 256, BN = 256, BK = 64, STAGES = 6;
+constexpr int BM = 256, BN = 256, STAGES = 6;
 constexpr int HM = BM / 2, HN = BN / 2;          // per-CTA halves
-constexpr int A_BYTES = HM * BK * 2;            // 16 KiB
-constexpr int B_BYTES = HN * BK * 2;            // 16 KiB
+constexpr int A_BYTES = HM * tc::KB_BYTES;      // 16 KiB
+constexpr int B_BYTES = HN * tc::KB_BYTES;      // 16 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512;
 constexpr int NTHREADS = 192;
@@ -270,6 +304,8 @@ constexpr uint32_t TMEM_COLS = 512;             // 2 accumulators x 256 f32 colu
 constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;     // shared::cluster address of the leader's copy
 
 using tc::Params;
+using tc::Geo;
+using tc::scale_exp2;
 using tc::fence_after;
 using tc::fence_before;
 using tc::mbar_expect_tx;
@@ -296,13 +332,21 @@ __device__ __forceinline__ void tma_load_2sm(void *dst, const CUtensorMap *map, 
       "l"((uint64_t)map), "r"(smem_u32(bar) & PEER_MASK), "r"(c0), "r"(c1)
       : "memory");
 }
+template <int ES>
 __device__ __forceinline__ void umma2(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   const uint32_t z = 0;
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, {%5, %5, %5, %5, %5, %5, %5, %5}, p;\n\t}" ::"r"(tmem_d),
-      "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(z));
+  if constexpr (ES == 2)
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, {%5, %5, %5, %5, %5, %5, %5, %5}, p;\n\t}" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(z));
+  else
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::f8f6f4 [%0], %1, %2, %3, {%5, %5, %5, %5, %5, %5, %5, %5}, p;\n\t}" ::"r"(tmem_d),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(z));
 }
 __device__ __forceinline__ void commit_both(uint64_t *bar) {
   asm volatile(
@@ -336,9 +380,12 @@ struct Sched {
   }
 };
 
+template <int ES>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
                     Params p, Sched sch) {
+  using G = Geo<ES>;
+  constexpr int BK = G::BK;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t *sA = smem;
@@ -393,20 +440,22 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
           const int k0 = kb * BK;
           uint8_t *a = sA + s * A_BYTES;
           if (!p.a_mn_major) {
-            tma_load_2sm(a, &tma_a, &full[s], k0, am);                    // box {64 K, 128 M}
+            tma_load_2sm(a, &tma_a, &full[s], k0, am);                    // box {BK, 128 M}
           } else {
-            tma_load_2sm(a, &tma_a, &full[s], am, k0);                    // box {64 M, 64 K} x 2
-            tma_load_2sm(a + tc::BOX_BYTES, &tma_a, &full[s], am + 64, k0);
+#pragma unroll
+            for (int q = 0; q < HM / G::MN_BOX; q++)                      // box {MN_BOX M, BK}
+              tma_load_2sm(a + q * G::BOX_BYTES, &tma_a, &full[s], am + G::MN_BOX * q, k0);
           }
           uint8_t *b = sB + s * B_BYTES;
-          tma_load_2sm(b, &tma_b, &full[s], bn, k0);                      // box {64 N, 64 K} x 2
-          tma_load_2sm(b + tc::BOX_BYTES, &tma_b, &full[s], bn + 64, k0);
+#pragma unroll
+          for (int q = 0; q < HN / G::MN_BOX; q++)                        // box {MN_BOX N, BK}
+            tma_load_2sm(b + q * G::BOX_BYTES, &tma_b, &full[s], bn + G::MN_BOX * q, k0);
         }
       }
     }
   } else if (warp == 1) {
     if (leader && lane == 0) {   // ---- MMA issuer (leader CTA, single thread)
-      const uint32_t idesc = (1u << 4) | (p.ab_fmt << 7) | (p.ab_fmt << 10) |
+      const uint32_t idesc = (1u << 4) | (p.a_fmt << 7) | (p.b_fmt << 10) |
                              ((uint32_t)p.a_mn_major << 15) | (1u << 16) |
                              ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
       int64_t cursor = cluster;
@@ -423,11 +472,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
           fence_after();
           const uint32_t abase = smem_u32(sA + s * A_BYTES), bbase = smem_u32(sB + s * B_BYTES);
 #pragma unroll
-          for (int kk = 0; kk < BK / 16; kk++) {
-            const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * 2048, tc::BOX_BYTES, 1024)
+          for (int kk = 0; kk < BK / G::MMA_K; kk++) {
+            const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * G::MN_STEP, G::BOX_BYTES, 1024)
                                              : umma_desc(abase + kk * 32, 16, 1024);
-            const uint64_t bd = umma_desc(bbase + kk * 2048, tc::BOX_BYTES, 1024);
-            umma2(dcol, ad, bd, idesc, (kb | kk) != 0);
+            const uint64_t bd = umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
+            umma2<ES>(dcol, ad, bd, idesc, (kb | kk) != 0);
           }
           commit_both(&empty[s]);   // stage s free in both CTAs once these MMAs retire
         }
@@ -437,6 +486,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
     }
   } else {   // ------------------------- epilogue warps 2..5 (both CTAs)
     const int q = warp & 3;
+    const int kab = scale_exp2(p);
     int64_t cursor = cluster;
     int m0, n0;
     uint32_t j = 0;
@@ -454,6 +504,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
             const int64_t col = (int64_t)n0 + cc * 16 + e;
             if (col >= p.N) break;
             float r = __uint_as_float(v[e]);
+            if (ES == 1) r = scalbnf(r, kab);   // exact power-of-two scale
             const int64_t idx = row * p.ldc + col;
             if (p.epi == EPI_AXPBY) r = __fmaf_rn(p.alpha, r, p.beta * load_c(p.Cin, p.cin_type, idx));
             else if (p.epi == EPI_DIV) r = r / p.div;
@@ -492,62 +543,74 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-// 2-D fp16 tensor map: inner (contiguous) extent, outer extent, outer stride in bytes,
-// box {64, box_outer}, 128-byte swizzle, zero fill out of bounds.
+// 2-D tensor map: inner (contiguous) extent, outer extent, outer stride in bytes,
+// box {128 bytes of elements, box_outer}, 128-byte swizzle, zero fill out of bounds.
 static bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer,
-                     uint64_t stride_bytes, uint32_t box_outer, bool bf16) {
+                     uint64_t stride_bytes, uint32_t box_outer, int type) {
   auto fn = encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {inner, outer};
   cuuint64_t strides[1] = {stride_bytes};
-  cuuint32_t box[2] = {64, box_outer};
+  cuuint32_t box[2] = {(cuuint32_t)(128 / dtype_size(type)), box_outer};
   cuuint32_t es[2] = {1, 1};
-  return fn(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
+  const CUtensorMapDataType dt = type == PS_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                 : type == PS_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                                  : CU_TENSOR_MAP_DATA_TYPE_UINT8;
+  return fn(m, dt, 2, const_cast<void *>(base), dims, strides, box, es,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 bool gemm_tc_supported(const GemmArgs &g) {
-  // both multiplicands fp16, or both bf16 (kind::f16 takes either, not a mix)
-  if (!((g.A.type == PS_F16 && g.B.type == PS_F16) || (g.A.type == PS_BF16 && g.B.type == PS_BF16)) ||
+  // both multiplicands fp16, or both bf16 (kind::f16 takes either, not a mix), or
+  // both fp8 (kind::f8f6f4: E4M3 / E5M2 in any mix)
+  const bool f8 = is_fp8(g.A.type) && is_fp8(g.B.type);
+  if (!((g.A.type == PS_F16 && g.B.type == PS_F16) || (g.A.type == PS_BF16 && g.B.type == PS_BF16) || f8) ||
       g.T != PS_F32)
     return false;
   if (g.c_type == PS_F64 || (g.epi == EPI_AXPBY && g.cin_type == PS_F64)) return false;
+  if (is_fp8(g.c_type) || (g.epi == EPI_AXPBY && is_fp8(g.cin_type))) return false;
+  if (f8 && (!g.A.sc || !g.B.sc)) return false;
   if (g.M <= 0 || g.N <= 0 || g.K <= 0 || g.M > (1 << 30) || g.N > (1 << 30) || g.K > (1 << 30))
     return false;
   if ((uintptr_t)g.A.p % 16 || (uintptr_t)g.B.p % 16) return false;
-  const bool a_k = g.A.s_col == 1 && (g.A.s_row * 2) % 16 == 0;    // row-major A
-  const bool a_m = g.A.s_row == 1 && (g.A.s_col * 2) % 16 == 0;    // SYRK data^T
-  const bool b_n = g.B.s_col == 1 && (g.B.s_row * 2) % 16 == 0;    // row-major B
+  const int64_t es = (int64_t)dtype_size(g.A.type);
+  const bool a_k = g.A.s_col == 1 && (g.A.s_row * es) % 16 == 0;    // row-major A
+  const bool a_m = g.A.s_row == 1 && (g.A.s_col * es) % 16 == 0;    // SYRK data^T
+  const bool b_n = g.B.s_col == 1 && (g.B.s_row * es) % 16 == 0;    // row-major B
   if (!(a_k || a_m) || !b_n) return false;
   return encode_fn() != nullptr;
 }
 
-ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
+template <int ES>
+static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   using namespace tc;
+  using G = Geo<ES>;
   static bool attr_set = false;
   if (!attr_set) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES));
+    PS_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES));
     attr_set = true;
   }
   CUtensorMap ma, mb;
   const bool a_mn = !(g.A.s_col == 1);
   bool ok;
-  const bool bf = g.A.type == PS_BF16;
-  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * 2, BM, bf);
-  else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * 2, 64, bf);
-  ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * 2, 64, bf);
+  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * ES, BM, g.A.type);
+  else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * ES, G::BK, g.A.type);
+  ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * ES, G::BK, g.B.type);
   if (!ok) {
     set_error("cuTensorMapEncodeTiled failed");
     return PS_ERR_CUDA;
   }
+  const uint32_t af = (g.A.type == PS_BF16 || g.A.type == PS_E5M2) ? 1u : 0u;
+  const uint32_t bfm = (g.B.type == PS_BF16 || g.B.type == PS_E5M2) ? 1u : 0u;
   Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
-           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, bf ? 1u : 0u};
+           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, af, bfm,
+           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr};
   if ((g.M > BM || g.N > BN) && !getenv("PS_TC_1SM")) {   // 2-CTA persistent path
     using namespace tc2;
     static bool attr2 = false;
     if (!attr2) {
-      PS_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+      PS_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel<ES>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    tc2::SMEM_BYTES));
       attr2 = true;
     }
@@ -562,14 +625,18 @@ ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
     int64_t clusters = num_sms() / 2;
     if (clusters > work) clusters = work;
     if (clusters < 1) clusters = 1;
-    gemm_tc2_kernel<<<(unsigned)(2 * clusters), tc2::NTHREADS, tc2::SMEM_BYTES, st>>>(ma, mb, p, sch);
+    gemm_tc2_kernel<ES><<<(unsigned)(2 * clusters), tc2::NTHREADS, tc2::SMEM_BYTES, st>>>(ma, mb, p, sch);
     PS_CHECK_LAUNCH("gemm_tc2_kernel");
     return PS_OK;
   }
   dim3 grid((unsigned)((g.N + BN - 1) / BN), (unsigned)((g.M + BM - 1) / BM));
-  gemm_tc_kernel<<<grid, NTHREADS, SMEM_BYTES, st>>>(ma, mb, p);
+  gemm_tc_kernel<ES><<<grid, NTHREADS, SMEM_BYTES, st>>>(ma, mb, p);
   PS_CHECK_LAUNCH("gemm_tc_kernel");
   return PS_OK;
+}
+
+ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
+  return is_fp8(g.A.type) ? gemm_tc_launch<1>(g, st) : gemm_tc_launch<2>(g, st);
 }
 
 }  // namespace ps

@@ -6,6 +6,13 @@ namespace ps {
 
 // ------------------------------------------------------------ conversion (a2)
 ps_status convert_async(const void *src, int st, void *dst, int dt, size_t n, cudaStream_t stream);
+// fp8 objects (reading #29, fp8.cu): encode with a fresh per-tensor scale computed
+// into *sc (sc == nullptr: unscaled, k = 0), decode with sc->k (nullptr: k = 0)
+constexpr int FP8_KMIN = -126, FP8_KMAX = 126;
+ps_status fp8_encode_async(const void *src, int st, void *dst, int dt, size_t n, ps_fp8_scale *sc,
+                           cudaStream_t stream);
+ps_status fp8_decode_async(const void *src, int st, void *dst, int dt, size_t n, const ps_fp8_scale *sc,
+                           cudaStream_t stream);
 // host-side f32 -> dt conversion (host_convert.cpp; Fig. 3a/3b)
 void host_convert_f32(const float *src, void *dst, int dt, size_t n, int threads, bool simd);
 
@@ -29,6 +36,7 @@ struct MatDesc {
   const void *p;
   int type;
   int64_t s_row, s_col;
+  const ps_fp8_scale *sc = nullptr;   // fp8 operand: its per-tensor scale record (reading #29)
 };
 enum Epilogue { EPI_PLAIN = 0, EPI_AXPBY = 1 /* fma(alpha, acc, beta*Cin) */, EPI_DIV = 2 };
 struct GemmArgs {
@@ -78,9 +86,11 @@ ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64
 // 3DCONV 27-point stencil (reading #26) on NI x NJ x NK
 ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
                        cudaStream_t st);
-// one FDTD-2D time step t (reading #27): ey, ex, hz passes
-ps_status fdtd2d_step_async(const void *fict, int tf, void *ex, int tex, void *ey, int tey, void *hz,
-                            int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st);
+// one statement of FDTD-2D time step t (reading #27): FDTD_EY = ey row 0 from fict and
+// the ey update in one pass; FDTD_EY0 / FDTD_EY1 = those two parts alone (reading #29)
+enum FdtdPart { FDTD_EY = 0, FDTD_EY0 = 1, FDTD_EY1 = 2, FDTD_EX = 3, FDTD_HZ = 4 };
+ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int tex, void *ey, int tey,
+                            void *hz, int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st);
 ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
                        int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
                        double eps, void *partial, cudaStream_t st);

@@ -47,6 +47,16 @@ template <> struct Deliver<BF16> {
   static __device__ __forceinline__ double exact(uint16_t h) { return (double)bf16_to_f32(h); }
 };
 
+// fp8 codes without a scale (ps_quality; the app path decodes scaled objects first)
+template <> struct Deliver<E4M3> {
+  static __device__ __forceinline__ float f(uint8_t q) { return canon_f32(fp8_to_f32(q, true)); }
+  static __device__ __forceinline__ double exact(uint8_t q) { return (double)fp8_to_f32(q, true); }
+};
+template <> struct Deliver<E5M2> {
+  static __device__ __forceinline__ float f(uint8_t q) { return canon_f32(fp8_to_f32(q, false)); }
+  static __device__ __forceinline__ double exact(uint8_t q) { return (double)fp8_to_f32(q, false); }
+};
+
 __device__ __forceinline__ void block_reduce3(double &sum, double &mx, unsigned long long &nf,
                                               double *s_sum, double *s_mx,
                                               unsigned long long *s_nf) {
@@ -161,7 +171,7 @@ int qblocks(size_t n) {
 ps_status backconv_quality_async(const void *out, int out_type, const double *ref, float *delivered,
                                  size_t n, QPart *parts, cudaStream_t st) {
   const int nb = qblocks(n);
-  return dispatch_store(out_type, [&](auto s) -> ps_status {
+  auto go = [&](auto s) -> ps_status {
     using S = decltype(s);
     if (delivered)
       backconv_quality_kernel<S, true><<<nb, QTHREADS, 0, st>>>((const raw_t<S> *)out, ref,
@@ -171,7 +181,10 @@ ps_status backconv_quality_async(const void *out, int out_type, const double *re
                                                                 nullptr, n, parts);
     PS_CHECK_LAUNCH("backconv_quality_kernel");
     return PS_OK;
-  });
+  };
+  if (out_type == PS_E4M3) return go(E4M3());
+  if (out_type == PS_E5M2) return go(E5M2());
+  return dispatch_store(out_type, go);
 }
 
 ps_status quality_finalize_async(const QPart *parts, int nparts, QPart *res, cudaStream_t st) {

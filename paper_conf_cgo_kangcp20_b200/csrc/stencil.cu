@@ -328,12 +328,13 @@ template <class SF, class SE, class SH>
 __global__ void __launch_bounds__(FD_NT) fdtd_ey_kernel(const raw_t<SF> *__restrict__ fict,
                                                         raw_t<SE> *__restrict__ ey,
                                                         const raw_t<SH> *__restrict__ hz, int64_t t,
-                                                        int64_t nx, int64_t ny) {
+                                                        int64_t nx, int64_t ny, int part) {
   using TA = T2<SF, SE>;   // ey[0][j] = fict[t]
   using TB = T2<SE, SH>;   // ey[i][j] -= 0.5 (hz[i][j] - hz[i-1][j])
   const int64_t jb = (int64_t)blockIdx.x * FD_COLS + threadIdx.x;
   for (int64_t i = blockIdx.y; i < nx; i += gridDim.y) {
     const int64_t row = i * ny;
+    if ((i == 0 && part == FDTD_EY1) || (i > 0 && part == FDTD_EY0)) continue;
     if (i == 0) {
       const TA f = ldg_t<SF, TA>(fict, t);
 #pragma unroll
@@ -419,25 +420,27 @@ __global__ void __launch_bounds__(FD_NT) fdtd_hz_kernel(raw_t<SH> *__restrict__ 
   }
 }
 
-ps_status fdtd2d_step_async(const void *fict, int tf, void *ex, int tex, void *ey, int tey, void *hz,
-                            int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st) {
+ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int tex, void *ey, int tey,
+                            void *hz, int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st) {
   if (nx <= 0 || ny <= 0) return PS_OK;
-  const dim3 grid((unsigned)((ny + FD_COLS - 1) / FD_COLS), (unsigned)(nx < 65535 ? nx : 65535));
-  ps_status s = dispatch_store(tf, [&](auto a) -> ps_status {
+  const int64_t rows = part == FDTD_EY0 ? 1 : nx;
+  if (part == FDTD_EY0) thz = PS_F32;   // the row-0 assignment reads fict only (hz unused)
+  if (part == FDTD_EY1) tf = PS_F32;    // the update reads hz only (fict unused)
+  const dim3 grid((unsigned)((ny + FD_COLS - 1) / FD_COLS), (unsigned)(rows < 65535 ? rows : 65535));
+  if (part <= FDTD_EY1) return dispatch_store(tf, [&](auto a) -> ps_status {
     return dispatch_store(tey, [&](auto b) -> ps_status {
       return dispatch_store(thz, [&](auto c) -> ps_status {
         using SF = decltype(a);
         using SE = decltype(b);
         using SH = decltype(c);
         fdtd_ey_kernel<SF, SE, SH><<<grid, FD_NT, 0, st>>>((const raw_t<SF> *)fict, (raw_t<SE> *)ey,
-                                                           (const raw_t<SH> *)hz, t, nx, ny);
+                                                           (const raw_t<SH> *)hz, t, nx, ny, part);
         PS_CHECK_LAUNCH("fdtd_ey_kernel");
         return PS_OK;
       });
     });
   });
-  if (s != PS_OK) return s;
-  s = dispatch_store(tex, [&](auto a) -> ps_status {
+  if (part == FDTD_EX) return dispatch_store(tex, [&](auto a) -> ps_status {
     return dispatch_store(thz, [&](auto c) -> ps_status {
       using SE = decltype(a);
       using SH = decltype(c);
@@ -446,7 +449,6 @@ ps_status fdtd2d_step_async(const void *fict, int tf, void *ex, int tex, void *e
       return PS_OK;
     });
   });
-  if (s != PS_OK) return s;
   return dispatch_store(thz, [&](auto a) -> ps_status {
     return dispatch_store(tex, [&](auto b) -> ps_status {
       return dispatch_store(tey, [&](auto c) -> ps_status {
