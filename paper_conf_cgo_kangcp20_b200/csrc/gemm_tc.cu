@@ -37,7 +37,12 @@ constexpr int KB_BYTES = 128;                   // one k-block = one 128-byte sw
 constexpr int A_BYTES = BM * KB_BYTES;          // 16 KiB
 constexpr int B_BYTES = BN * KB_BYTES;          // 32 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+// epilogue staging: each of the 4 epilogue warps turns a 32 x 32 accumulator chunk
+// (thread = row, from tcgen05.ld.32x32b) into coalesced row segments through smem
+constexpr int EPI_COLS = 32;
+constexpr int EPI_STRIDE = 36;                                // floats per staged row (conflict-free float4)
+constexpr int EPI_SMEM = 4 * 32 * EPI_STRIDE * 4;             // 18 KiB
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + EPI_SMEM;
 constexpr int NTHREADS = 192;
 constexpr uint32_t TMEM_COLS = 256;
 // element-size dependent geometry (ES = 2: f16/bf16, ES = 1: fp8)
@@ -52,6 +57,7 @@ template <int ES> struct Geo {
 struct Params {
   int M, N, K;
   int a_mn_major;
+  int b_k_major;     // B(k, j) K-contiguous (a transposed copy) instead of N-major
   void *C;
   int c_type;
   int64_t ldc;
@@ -62,6 +68,7 @@ struct Params {
   int upper_only;
   uint32_t a_fmt, b_fmt;   // kind::f16: 0 = f16, 1 = bf16 (reading #28); kind::f8f6f4: 0 = E4M3, 1 = E5M2
   const ps_fp8_scale *sa, *sb;   // fp8 operands: per-tensor scales (reading #29)
+  int vec4;                // C / Cin rows 4-element aligned: vector epilogue stores / loads
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -150,6 +157,19 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+        "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+        "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]),
+        "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]),
+        "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
 __device__ __forceinline__ float load_c(const void *p, int type, int64_t idx) {
   if (type == PS_F32) return ((const float *)p)[idx];
   const uint16_t h = ((const uint16_t *)p)[idx];
@@ -159,6 +179,87 @@ __device__ __forceinline__ void store_c(void *p, int type, int64_t idx, float v)
   if (type == PS_F32) ((float *)p)[idx] = v;
   else if (type == PS_BF16) ((uint16_t *)p)[idx] = rne_bf16(v);
   else ((uint16_t *)p)[idx] = rne_f16(v);
+}
+
+__device__ __forceinline__ float epi_op(const Params &p, float r, float cin) {
+  if (p.epi == EPI_AXPBY) return __fmaf_rn(p.alpha, r, p.beta * cin);
+  if (p.epi == EPI_DIV) return r / p.div;
+  return r;
+}
+
+// Epilogue of one 32-row x 32-column accumulator chunk held by this warp (lane =
+// row row0 + lane, v = columns col0..col0+31 from tcgen05.ld.32x32b.x32): staged
+// through smem, then written as coalesced row segments -- lane l handles row
+// 4i + l/8 and columns 4(l%8)..+3 (one 16-byte f32 or 8-byte 16-bit access, and
+// the matching Cin load for alpha/beta).  fp8 operands: accumulator x 2^kab first.
+__device__ __forceinline__ void epi_chunk(const Params &p, float *stg, int lane, int64_t row0,
+                                          int64_t col0, const uint32_t (&v)[32], int kab) {
+  float4 *srow = reinterpret_cast<float4 *>(stg + lane * EPI_STRIDE);
+#pragma unroll
+  for (int q = 0; q < 8; q++)
+    srow[q] = make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]),
+                          __uint_as_float(v[4 * q + 2]), __uint_as_float(v[4 * q + 3]));
+  __syncwarp();
+  const int cq = lane & 7;
+  const int64_t col = col0 + cq * 4;
+  const bool vcol = p.vec4 && col + 3 < p.N;
+  // 1) the chunk's 8 Cin segments of this lane, all loads in flight at once (alpha/beta)
+  float c[8][4];
+#pragma unroll
+  for (int i = 0; i < 8; i++) {
+    c[i][0] = c[i][1] = c[i][2] = c[i][3] = 0.f;
+    const int64_t row = row0 + i * 4 + (lane >> 3);
+    if (p.epi != EPI_AXPBY || row >= p.M) continue;
+    const int64_t idx = row * p.ldc + col;
+    if (vcol) {
+      if (p.cin_type == PS_F32) {
+        const float4 t = __ldg(reinterpret_cast<const float4 *>((const float *)p.Cin + idx));
+        c[i][0] = t.x; c[i][1] = t.y; c[i][2] = t.z; c[i][3] = t.w;
+      } else {
+        const uint2 t = __ldg(reinterpret_cast<const uint2 *>((const uint16_t *)p.Cin + idx));
+        const uint16_t h[4] = {(uint16_t)(t.x & 0xFFFF), (uint16_t)(t.x >> 16), (uint16_t)(t.y & 0xFFFF),
+                               (uint16_t)(t.y >> 16)};
+#pragma unroll
+        for (int e = 0; e < 4; e++) c[i][e] = p.cin_type == PS_BF16 ? bf16_to_f32(h[e]) : f16_to_f32(h[e]);
+      }
+    } else {
+#pragma unroll
+      for (int e = 0; e < 4; e++)
+        if (col + e < p.N) c[i][e] = load_c(p.Cin, p.cin_type, idx + e);
+    }
+  }
+  // 2) scale, epilogue op, RNE store (R1) as coalesced row segments
+#pragma unroll
+  for (int i = 0; i < 8; i++) {
+    const int r = i * 4 + (lane >> 3);
+    const int64_t row = row0 + r;
+    const float4 a = *reinterpret_cast<const float4 *>(stg + r * EPI_STRIDE + cq * 4);
+    float x[4] = {a.x, a.y, a.z, a.w};
+    if (row >= p.M) continue;
+    if (kab) {
+#pragma unroll
+      for (int e = 0; e < 4; e++) x[e] = scalbnf(x[e], kab);   // exact power-of-two scale
+    }
+#pragma unroll
+    for (int e = 0; e < 4; e++) x[e] = epi_op(p, x[e], c[i][e]);
+    const int64_t idx = row * p.ldc + col;
+    if (vcol) {
+      if (p.c_type == PS_F32) {
+        *reinterpret_cast<float4 *>((float *)p.C + idx) = make_float4(x[0], x[1], x[2], x[3]);
+      } else {
+        uint16_t h[4];
+#pragma unroll
+        for (int e = 0; e < 4; e++) h[e] = p.c_type == PS_BF16 ? rne_bf16(x[e]) : rne_f16(x[e]);
+        *reinterpret_cast<uint2 *>((uint16_t *)p.C + idx) =
+            make_uint2((uint32_t)h[0] | ((uint32_t)h[1] << 16), (uint32_t)h[2] | ((uint32_t)h[3] << 16));
+      }
+    } else {
+#pragma unroll
+      for (int e = 0; e < 4; e++)
+        if (col + e < p.N) store_c(p.C, p.c_type, idx + e, x[e]);
+    }
+  }
+  __syncwarp();
 }
 
 template <int ES>
@@ -175,6 +276,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   uint64_t *empty = full + STAGES;
   uint64_t *tfull = empty + STAGES;
   uint32_t *tmem_slot = (uint32_t *)(tfull + 1);
+  float *epi_stage = (float *)(smem + STAGES * STAGE_BYTES + 256);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
@@ -219,9 +321,13 @@ __global__ void __launch_bounds__(NTHREADS, 1)
             tma_load_2d(a + q * G::BOX_BYTES, &tma_a, &full[s], m0 + G::MN_BOX * q, k0);
         }
         uint8_t *b = sB + s * B_BYTES;
+        if (p.b_k_major) {
+          tma_load_2d(b, &tma_b, &full[s], k0, n0);                 // box {BK, 256 N}
+        } else {
 #pragma unroll
-        for (int q = 0; q < BN / G::MN_BOX; q++)
-          tma_load_2d(b + q * G::BOX_BYTES, &tma_b, &full[s], n0 + G::MN_BOX * q, k0);
+          for (int q = 0; q < BN / G::MN_BOX; q++)
+            tma_load_2d(b + q * G::BOX_BYTES, &tma_b, &full[s], n0 + G::MN_BOX * q, k0);
+        }
       }
     }
   } else if (warp == 1) {
@@ -229,7 +335,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       const uint32_t idesc = (1u << 4)                          // D = f32
                              | (p.a_fmt << 7) | (p.b_fmt << 10)     // A, B format
                              | ((uint32_t)p.a_mn_major << 15)   // A major
-                             | (1u << 16)                       // B is N-major
+                             | ((uint32_t)(!p.b_k_major) << 16) // B major
                              | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
       for (int kb = 0; kb < nk; kb++) {
         const int s = kb % STAGES;
@@ -243,7 +349,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           // MN-major SW128: +MMA_K K-rows of 128 B; LBO = one MN box between boxes.
           const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * G::MN_STEP, G::BOX_BYTES, 1024)
                                            : umma_desc(abase + kk * 32, 16, 1024);
-          const uint64_t bd = umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
+          const uint64_t bd = p.b_k_major ? umma_desc(bbase + kk * 32, 16, 1024)
+                                          : umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
           umma_f16<ES>(tmem, ad, bd, idesc, (kb | kk) != 0);
         }
         umma_commit(&empty[s]);   // frees the stage when these MMAs retire
@@ -255,23 +362,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     fence_after();
     const int kab = scale_exp2(p);
     const int q = warp & 3;                 // TMEM lane quarter this warp may access
-    const int64_t row = (int64_t)m0 + q * 32 + lane;
-    for (int cc = 0; cc < BN / 16; cc++) {
-      uint32_t v[16];
-      tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * 16), v);
-      if (row < p.M) {
-#pragma unroll
-        for (int e = 0; e < 16; e++) {
-          const int64_t col = (int64_t)n0 + cc * 16 + e;
-          if (col >= p.N) break;
-          float r = __uint_as_float(v[e]);
-          if (ES == 1) r = scalbnf(r, kab);   // exact power-of-two scale
-          const int64_t idx = row * p.ldc + col;
-          if (p.epi == EPI_AXPBY) r = __fmaf_rn(p.alpha, r, p.beta * load_c(p.Cin, p.cin_type, idx));
-          else if (p.epi == EPI_DIV) r = r / p.div;
-          store_c(p.C, p.c_type, idx, r);
-        }
-      }
+    float *stg = epi_stage + (warp - 2) * 32 * EPI_STRIDE;
+    for (int cc = 0; cc < BN / EPI_COLS; cc++) {
+      if ((int64_t)n0 + cc * EPI_COLS >= p.N) break;
+      uint32_t v[32];
+      tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
+      epi_chunk(p, stg, lane, (int64_t)m0 + q * 32, (int64_t)n0 + cc * EPI_COLS, v, kab);
     }
   }
   fence_before();
@@ -298,7 +394,7 @@ constexpr int HM = BM / 2, HN = BN / 2;          // per-CTA halves
 constexpr int A_BYTES = HM * tc::KB_BYTES;      // 16 KiB
 constexpr int B_BYTES = HN * tc::KB_BYTES;      // 16 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512 + tc::EPI_SMEM;
 constexpr int NTHREADS = 192;
 constexpr uint32_t TMEM_COLS = 512;             // 2 accumulators x 256 f32 columns
 constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;     // shared::cluster address of the leader's copy
@@ -313,6 +409,10 @@ using tc::mbar_init;
 using tc::mbar_wait;
 using tc::smem_u32;
 using tc::tmem_ld16;
+using tc::tmem_ld32;
+using tc::epi_chunk;
+using tc::EPI_COLS;
+using tc::EPI_STRIDE;
 using tc::umma_desc;
 using tc::load_c;
 using tc::store_c;
@@ -395,6 +495,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
   uint64_t *tfull = empty + STAGES;      // [2]
   uint64_t *tempty = tfull + 2;          // [2]
   uint32_t *tmem_slot = (uint32_t *)(tempty + 2);
+  float *epi_stage = (float *)(smem + STAGES * STAGE_BYTES + 512);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_rank();
@@ -447,16 +548,20 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
               tma_load_2sm(a + q * G::BOX_BYTES, &tma_a, &full[s], am + G::MN_BOX * q, k0);
           }
           uint8_t *b = sB + s * B_BYTES;
+          if (p.b_k_major) {
+            tma_load_2sm(b, &tma_b, &full[s], k0, bn);                    // box {BK, 128 N}
+          } else {
 #pragma unroll
-          for (int q = 0; q < HN / G::MN_BOX; q++)                        // box {MN_BOX N, BK}
-            tma_load_2sm(b + q * G::BOX_BYTES, &tma_b, &full[s], bn + G::MN_BOX * q, k0);
+            for (int q = 0; q < HN / G::MN_BOX; q++)                      // box {MN_BOX N, BK}
+              tma_load_2sm(b + q * G::BOX_BYTES, &tma_b, &full[s], bn + G::MN_BOX * q, k0);
+          }
         }
       }
     }
   } else if (warp == 1) {
     if (leader && lane == 0) {   // ---- MMA issuer (leader CTA, single thread)
       const uint32_t idesc = (1u << 4) | (p.a_fmt << 7) | (p.b_fmt << 10) |
-                             ((uint32_t)p.a_mn_major << 15) | (1u << 16) |
+                             ((uint32_t)p.a_mn_major << 15) | ((uint32_t)(!p.b_k_major) << 16) |
                              ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
       int64_t cursor = cluster;
       int m0, n0;
@@ -475,7 +580,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
           for (int kk = 0; kk < BK / G::MMA_K; kk++) {
             const uint64_t ad = p.a_mn_major ? umma_desc(abase + kk * G::MN_STEP, G::BOX_BYTES, 1024)
                                              : umma_desc(abase + kk * 32, 16, 1024);
-            const uint64_t bd = umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
+            const uint64_t bd = p.b_k_major ? umma_desc(bbase + kk * 32, 16, 1024)
+                                            : umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
             umma2<ES>(dcol, ad, bd, idesc, (kb | kk) != 0);
           }
           commit_both(&empty[s]);   // stage s free in both CTAs once these MMAs retire
@@ -494,23 +600,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
       const uint32_t acc = j & 1u;
       mbar_wait(&tfull[acc], (j >> 1) & 1u);
       fence_after();
-      const int64_t row = (int64_t)m0 + rank * HM + q * 32 + lane;
-      for (int cc = 0; cc < BN / 16; cc++) {
-        uint32_t v[16];
-        tmem_ld16(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * 16), v);
-        if (row < p.M) {
-#pragma unroll
-          for (int e = 0; e < 16; e++) {
-            const int64_t col = (int64_t)n0 + cc * 16 + e;
-            if (col >= p.N) break;
-            float r = __uint_as_float(v[e]);
-            if (ES == 1) r = scalbnf(r, kab);   // exact power-of-two scale
-            const int64_t idx = row * p.ldc + col;
-            if (p.epi == EPI_AXPBY) r = __fmaf_rn(p.alpha, r, p.beta * load_c(p.Cin, p.cin_type, idx));
-            else if (p.epi == EPI_DIV) r = r / p.div;
-            store_c(p.C, p.c_type, idx, r);
-          }
-        }
+      const int64_t row0 = (int64_t)m0 + rank * HM + q * 32;
+      float *stg = epi_stage + (warp - 2) * 32 * EPI_STRIDE;
+      for (int cc = 0; cc < BN / EPI_COLS; cc++) {
+        if ((int64_t)n0 + cc * EPI_COLS >= p.N) break;
+        uint32_t v[32];
+        tmem_ld32(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
+        epi_chunk(p, stg, lane, row0, (int64_t)n0 + cc * EPI_COLS, v, kab);
       }
       fence_before();
       __syncwarp();
@@ -578,7 +674,8 @@ bool gemm_tc_supported(const GemmArgs &g) {
   const bool a_k = g.A.s_col == 1 && (g.A.s_row * es) % 16 == 0;    // row-major A
   const bool a_m = g.A.s_row == 1 && (g.A.s_col * es) % 16 == 0;    // SYRK data^T
   const bool b_n = g.B.s_col == 1 && (g.B.s_row * es) % 16 == 0;    // row-major B
-  if (!(a_k || a_m) || !b_n) return false;
+  const bool b_k = g.B.s_row == 1 && (g.B.s_col * es) % 16 == 0;    // K-contiguous B
+  if (!(a_k || a_m) || !(b_n || b_k)) return false;
   return encode_fn() != nullptr;
 }
 
@@ -593,20 +690,30 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   }
   CUtensorMap ma, mb;
   const bool a_mn = !(g.A.s_col == 1);
+  const bool b_k = !(g.B.s_col == 1);
+  const bool two = (g.M > BM || g.N > BN) && !getenv("PS_TC_1SM");
   bool ok;
   if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * ES, BM, g.A.type);
   else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * ES, G::BK, g.A.type);
-  ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * ES, G::BK, g.B.type);
+  if (!b_k) ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * ES, G::BK, g.B.type);
+  else ok = ok && make_map(&mb, g.B.p, (uint64_t)g.K, (uint64_t)g.N, (uint64_t)g.B.s_col * ES,
+                           two ? tc2::HN : BN, g.B.type);
   if (!ok) {
     set_error("cuTensorMapEncodeTiled failed");
     return PS_ERR_CUDA;
   }
   const uint32_t af = (g.A.type == PS_BF16 || g.A.type == PS_E5M2) ? 1u : 0u;
   const uint32_t bfm = (g.B.type == PS_BF16 || g.B.type == PS_E5M2) ? 1u : 0u;
-  Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
+  Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, b_k ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
            (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, af, bfm,
-           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr};
-  if ((g.M > BM || g.N > BN) && !getenv("PS_TC_1SM")) {   // 2-CTA persistent path
+           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr, 0};
+  {   // vector epilogue: rows of C (and Cin) start 16-byte (f32) / 8-byte (16-bit) aligned
+    const int64_t cb = (int64_t)dtype_size(g.c_type);
+    bool v4 = g.ldc % 4 == 0 && (uintptr_t)g.C % (4 * cb) == 0;
+    if (g.epi == EPI_AXPBY) v4 = v4 && (uintptr_t)g.Cin % (4 * dtype_size(g.cin_type)) == 0;
+    p.vec4 = v4 ? 1 : 0;
+  }
+  if (two) {   // 2-CTA persistent path
     using namespace tc2;
     static bool attr2 = false;
     if (!attr2) {
@@ -635,7 +742,43 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   return PS_OK;
 }
 
-ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
+// out[j * K + k] = in[k * ld + j]: an N-major K x N operand copied K-contiguous
+template <class E>
+__global__ void __launch_bounds__(256) transpose_kernel(const E *__restrict__ in, E *__restrict__ out,
+                                                        int64_t K, int64_t N, int64_t ld) {
+  __shared__ E t[32][33];
+  const int64_t k0 = (int64_t)blockIdx.y * 32, j0 = (int64_t)blockIdx.x * 32;
+  for (int r = threadIdx.y; r < 32; r += 8) {
+    const int64_t k = k0 + r, j = j0 + threadIdx.x;
+    if (k < K && j < N) t[r][threadIdx.x] = in[k * ld + j];
+  }
+  __syncthreads();
+  for (int r = threadIdx.y; r < 32; r += 8) {
+    const int64_t j = j0 + r, k = k0 + threadIdx.x;
+    if (k < K && j < N) out[j * K + k] = t[threadIdx.x][r];
+  }
+}
+
+ps_status gemm_tc_async(const GemmArgs &g0, cudaStream_t st) {
+  GemmArgs g = g0;
+  static const bool bt = getenv("PS_TC_BT") != nullptr;   // experiment: K-major B via a transposed copy
+  if (bt && g.B.s_col == 1 && g.K % 16 == 0) {
+    static void *buf = nullptr;
+    static size_t cap = 0;
+    const size_t es = dtype_size(g.B.type), need = (size_t)g.K * (size_t)g.N * es;
+    if (need > cap) {
+      if (buf) cudaFree(buf);
+      PS_CUDA(cudaMalloc(&buf, need));
+      cap = need;
+    }
+    const dim3 grid((unsigned)((g.N + 31) / 32), (unsigned)((g.K + 31) / 32)), blk(32, 8);
+    if (es == 1) transpose_kernel<uint8_t><<<grid, blk, 0, st>>>((const uint8_t *)g.B.p, (uint8_t *)buf, g.K, g.N, g.B.s_row);
+    else transpose_kernel<uint16_t><<<grid, blk, 0, st>>>((const uint16_t *)g.B.p, (uint16_t *)buf, g.K, g.N, g.B.s_row);
+    PS_CHECK_LAUNCH("transpose_kernel");
+    g.B.p = buf;
+    g.B.s_row = 1;
+    g.B.s_col = g.K;
+  }
   return is_fp8(g.A.type) ? gemm_tc_launch<1>(g, st) : gemm_tc_launch<2>(g, st);
 }
 
