@@ -8,12 +8,9 @@
 //     +0; slab value = xor butterfly 16..1 (a + partner); 8 slabs form a tile,
 //     slab values added left to right; tile values added left to right.
 //
-// One kernel shape serves every statement: a work unit is (256-row chunk,
-// 8-slab column tile); the units, numbered tile-major (a tile's chunks are
-// consecutive), are split into one contiguous range per CTA of a grid of
-// SMs x occupancy (8 warps each), so every resident slot streams down its
-// column band with the load balanced to one unit; warp w streams slab 8t+w,
-// one 16-byte load per lane per row (16 rows in flight), so each element of A is read
+// One kernel shape serves every statement: a CTA = 8 warps owns one 8-slab
+// column tile and walks 256-row chunks; warp w streams slab 8t+w, one 16-byte
+// load per lane per row (4 rows in flight), so each element of A is read
 // ONCE for the column sums AND the row dots.  BICG (s = A^T r, q = A p) is a
 // single pass over A.  Partials (chunk x columns, tile x rows) go to the
 // workspace and two tiny kernels finish them in order.  HBM-bound:
@@ -44,7 +41,6 @@ struct TileArgs {
   int64_t nchunks, ntiles, nslabs;
   int vec_ok;
 };
-// (the work-unit count is nchunks * ntiles; unit u = tile u / nchunks, chunk u % nchunks)
 
 template <class SA, class TC, class TR, int CM, bool RD>
 __global__ void __launch_bounds__(TTHREADS) tile_kernel(TileArgs a) {
@@ -56,30 +52,22 @@ __global__ void __launch_bounds__(TTHREADS) tile_kernel(TileArgs a) {
   __shared__ TR part[RD ? COLSUM_CHUNK : 1][TILE_SLABS + 1];
   __shared__ TC sw[CM == COL_DOT ? COLSUM_CHUNK : 1];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t nunits = a.nchunks * a.ntiles;
-  int64_t cur_tile = -1;
-  int64_t j0 = 0;
-  int nv = 0;
-  bool vec = false, wfull = false;
+  const int64_t tcol = blockIdx.x;
+  const int64_t j0 = (tcol * TILE_SLABS + warp) * (32 * V) + (int64_t)lane * V;
+  const int64_t rem = a.cols - j0;
+  const int nv = rem <= 0 ? 0 : (rem >= V ? V : (int)rem);
+  const bool vec = a.vec_ok && nv == V;
+  const bool wfull = __all_sync(0xffffffffu, vec);   // warp-uniform fast path
+
   TR xv[V];
   TC mu[V];
-
-  const int64_t u0 = nunits * blockIdx.x / gridDim.x, u1 = nunits * (blockIdx.x + 1) / gridDim.x;
-  for (int64_t u = u0; u < u1; u++) {
-    const int64_t tcol = u / a.nchunks, rc = u % a.nchunks;
-    if (tcol != cur_tile) {   // this column tile's lane columns and vector values
-      cur_tile = tcol;
-      j0 = (tcol * TILE_SLABS + warp) * (32 * V) + (int64_t)lane * V;
-      const int64_t rem = a.cols - j0;
-      nv = rem <= 0 ? 0 : (rem >= V ? V : (int)rem);
-      vec = a.vec_ok && nv == V;
-      wfull = __all_sync(0xffffffffu, vec);   // warp-uniform fast path
 #pragma unroll
-      for (int v = 0; v < V; v++) {
-        xv[v] = (RD && v < nv) ? load_any<TR>(a.x, a.tx, j0 + v) : TR(0);
-        mu[v] = (CM == COL_SQDEV && v < nv) ? load_any<TC>(a.w, a.tw, j0 + v) : TC(0);
-      }
-    }
+  for (int v = 0; v < V; v++) {
+    xv[v] = (RD && v < nv) ? load_any<TR>(a.x, a.tx, j0 + v) : TR(0);
+    mu[v] = (CM == COL_SQDEV && v < nv) ? load_any<TC>(a.w, a.tw, j0 + v) : TC(0);
+  }
+
+  for (int64_t rc = blockIdx.y; rc < a.nchunks; rc += gridDim.y) {
     const int64_t i0 = rc * COLSUM_CHUNK;
     const int64_t i1 = (a.rows < i0 + COLSUM_CHUNK) ? a.rows : i0 + COLSUM_CHUNK;
     if (CM == COL_DOT) {   // stage this chunk's w_i (T_c) in shared memory
@@ -240,9 +228,12 @@ static ps_status launch_tile(const TileArgs &a, cudaStream_t st) {
     if (occ < 1) occ = 1;
   }
   const int64_t cap = (int64_t)num_sms() * occ;
-  const int64_t units = a.nchunks * a.ntiles;
-  const int64_t grid = units < cap ? units : cap;   // persistent: every resident slot busy
-  tile_kernel<SA, TC, TR, CM, RD><<<(unsigned)grid, TTHREADS, 0, st>>>(a);
+  int64_t gy = cap / a.ntiles;
+  if (gy < 1) gy = 1;
+  if (gy > a.nchunks) gy = a.nchunks;
+  const int64_t per = (a.nchunks + gy - 1) / gy;   // equal chunk counts per CTA row
+  gy = (a.nchunks + per - 1) / per;
+  tile_kernel<SA, TC, TR, CM, RD><<<dim3((unsigned)a.ntiles, (unsigned)gy), TTHREADS, 0, st>>>(a);
   PS_CHECK_LAUNCH("tile_kernel");
   return PS_OK;
 }
