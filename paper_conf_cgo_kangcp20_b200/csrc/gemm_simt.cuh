@@ -20,11 +20,20 @@ namespace simt {
 
 template <class T> struct Cfg;
 // CH: consecutive columns per thread chunk (one 16-byte shared load); a thread's TN
-// columns are TN/CH chunks spaced 16*CH apart, so 8 lanes of a quarter-warp read 128
-// contiguous bytes of B (conflict-free for 8-byte T as well as 4-byte T)
-template <> struct Cfg<float> { static constexpr int BM = 128, BN = 128, BK = 16, TM = 8, TN = 8, CH = 4; };
-template <> struct Cfg<double> { static constexpr int BM = 128, BN = 128, BK = 8, TM = 8, TN = 8, CH = 2; };
-constexpr int THREADS = 256;
+// columns are TN/CH chunks spaced TX*CH apart, so 8 lanes of a quarter-warp read 128
+// contiguous bytes of B (conflict-free for 8-byte T as well as 4-byte T).  Threads:
+// TX along N x 16 along M; each owns TM = 8 rows (two runs of 4, BM/2 apart).
+// (Measured at 8192^3 on B200, f64: 256 threads x 8 x 8, BK = 8 -> 22.6 TFLOP/s; BK = 16
+// -> 20.9 (254 registers); 512 threads x 8 x 4, BK = 16 -> 21.1.)
+template <> struct Cfg<float> {
+  static constexpr int BM = 128, BN = 128, BK = 16, TM = 8, TN = 8, CH = 4, TX = 16, THREADS = 256;
+};
+template <> struct Cfg<double> {
+  static constexpr int BM = 128, BN = 128, BK = 8, TM = 8, TN = 8, CH = 2, TX = 16, THREADS = 256;
+};
+template <class T> constexpr int smem_bytes() {
+  return 2 * Cfg<T>::BK * (Cfg<T>::BM + Cfg<T>::BN) * (int)sizeof(T);
+}
 
 struct Params {
   int64_t M, N, K;
@@ -90,14 +99,17 @@ __device__ __forceinline__ void load_run(const raw_t<S> *p, T (&out)[E]) {
 }
 
 template <class T, class SA, class SB, bool AK>
-__global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta, T div) {
+__global__ void __launch_bounds__(Cfg<T>::THREADS, 1) gemm_kernel(Params p, T alpha, T beta, T div) {
   constexpr int BM = Cfg<T>::BM, BN = Cfg<T>::BN, BK = Cfg<T>::BK;
-  constexpr int TM = Cfg<T>::TM, TN = Cfg<T>::TN, CH = Cfg<T>::CH;
+  constexpr int TM = Cfg<T>::TM, TN = Cfg<T>::TN, CH = Cfg<T>::CH, TX = Cfg<T>::TX;
+  constexpr int THREADS = Cfg<T>::THREADS;
+  static_assert(TX * TN == BN && (THREADS / TX) * TM == BM, "thread tiling");
   constexpr int EA = BM * BK / THREADS, EB = BK * BN / THREADS;   // elements per thread per tile
-  __shared__ __align__(16) T As[2][BK][BM];
-  __shared__ __align__(16) T Bs[2][BK][BN];
+  extern __shared__ __align__(16) unsigned char smem_dyn[];
+  T(*As)[BK][BM] = reinterpret_cast<T(*)[BK][BM]>(smem_dyn);                      // [2][BK][BM]
+  T(*Bs)[BK][BN] = reinterpret_cast<T(*)[BK][BN]>(smem_dyn + 2 * BK * BM * sizeof(T));   // [2][BK][BN]
 
-  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int tid = threadIdx.x, tx = tid % TX, ty = tid / TX;
   const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
   if (p.upper_only && m0 + p.row_off >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
 
@@ -163,7 +175,7 @@ __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta
 #pragma unroll
       for (int i = 0; i < TM; i++) a[i] = As[buf][k][(i / 4) * (BM / 2) + ty * 4 + (i % 4)];
 #pragma unroll
-      for (int j = 0; j < TN; j++) b[j] = Bs[buf][k][(j / CH) * (16 * CH) + tx * CH + (j % CH)];
+      for (int j = 0; j < TN; j++) b[j] = Bs[buf][k][(j / CH) * (TX * CH) + tx * CH + (j % CH)];
 #pragma unroll
       for (int i = 0; i < TM; i++)
 #pragma unroll
@@ -183,7 +195,7 @@ __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta
     if (gm >= p.M) continue;
 #pragma unroll
     for (int j = 0; j < TN; j++) {
-      const int64_t gn = n0 + (j / CH) * (16 * CH) + tx * CH + (j % CH);
+      const int64_t gn = n0 + (j / CH) * (TX * CH) + tx * CH + (j % CH);
       if (gn >= p.N) continue;
       T r = acc[i][j];
       const int64_t idx = gm * p.ldc + gn;
@@ -197,10 +209,17 @@ __global__ void __launch_bounds__(THREADS) gemm_kernel(Params p, T alpha, T beta
 template <class T, class SA, class SB>
 ps_status launch(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
   using C = Cfg<T>;
+  constexpr int SM = smem_bytes<T>();
+  static bool attr = false;
+  if (!attr) {
+    PS_CUDA(cudaFuncSetAttribute(gemm_kernel<T, SA, SB, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
+    PS_CUDA(cudaFuncSetAttribute(gemm_kernel<T, SA, SB, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
+    attr = true;
+  }
   dim3 grid((unsigned)((p.N + C::BN - 1) / C::BN), (unsigned)((p.M + C::BM - 1) / C::BM));
   // scalars are RNE-rounded from their fp64 literal to T (R2); the host cast is RNE
-  if (ak) gemm_kernel<T, SA, SB, true><<<grid, THREADS, 0, st>>>(p, (T)alpha, (T)beta, (T)div);
-  else gemm_kernel<T, SA, SB, false><<<grid, THREADS, 0, st>>>(p, (T)alpha, (T)beta, (T)div);
+  if (ak) gemm_kernel<T, SA, SB, true><<<grid, C::THREADS, SM, st>>>(p, (T)alpha, (T)beta, (T)div);
+  else gemm_kernel<T, SA, SB, false><<<grid, C::THREADS, SM, st>>>(p, (T)alpha, (T)beta, (T)div);
   PS_CHECK_LAUNCH("gemm_simt_kernel");
   return PS_OK;
 }
