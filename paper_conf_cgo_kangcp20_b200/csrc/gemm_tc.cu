@@ -13,7 +13,7 @@
 //                      one lane issues tcgen05.mma.kind::f16 (M=128, N=256,
 //                      K=16) and tcgen05.commit frees each stage / signals
 //                      the epilogue
-//   warps 2..5       : epilogue -- tcgen05.ld 32x32b (warp w reads TMEM lanes
+//   warps 2..9       : epilogue -- tcgen05.ld 32x32b (warp w reads TMEM lanes
 //                      32*(w%4)..), alpha/beta or divide in f32, RNE store to
 //                      the output object's precision (R1)
 // A may be K-major (row-major A) or M-major (SYRK's data^T); B is N-major.
@@ -32,7 +32,7 @@
 namespace ps {
 namespace tc {
 
-constexpr int BM = 128, BN = 256, STAGES = 4;
+constexpr int BM = 128, BN = 256, STAGES = 3;
 constexpr int KB_BYTES = 128;                   // one k-block = one 128-byte swizzled row
 constexpr int A_BYTES = BM * KB_BYTES;          // 16 KiB
 constexpr int B_BYTES = BN * KB_BYTES;          // 32 KiB
@@ -41,9 +41,13 @@ constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 // (thread = row, from tcgen05.ld.32x32b) into coalesced row segments through smem
 constexpr int EPI_COLS = 32;
 constexpr int EPI_STRIDE = 36;                                // floats per staged row (conflict-free float4)
-constexpr int EPI_SMEM = 4 * 32 * EPI_STRIDE * 4;             // 18 KiB
+// 8 epilogue warps: two per TMEM lane quarter (warp w may read lanes 32 (w % 4)..),
+// each draining half of the accumulator's columns -- twice the memory-level
+// parallelism of one warp per quarter, which paced the fp8 tiles (ncu / PS_TC_NOEPI)
+constexpr int EPI_WARPS = 8;
+constexpr int EPI_SMEM = EPI_WARPS * 32 * EPI_STRIDE * 4;     // 36 KiB
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + EPI_SMEM;
-constexpr int NTHREADS = 192;
+constexpr int NTHREADS = 64 + 32 * EPI_WARPS;
 constexpr uint32_t TMEM_COLS = 256;
 // element-size dependent geometry (ES = 2: f16/bf16, ES = 1: fp8)
 template <int ES> struct Geo {
@@ -69,6 +73,7 @@ struct Params {
   uint32_t a_fmt, b_fmt;   // kind::f16: 0 = f16, 1 = bf16 (reading #28); kind::f8f6f4: 0 = E4M3, 1 = E5M2
   const ps_fp8_scale *sa, *sb;   // fp8 operands: per-tensor scales (reading #29)
   int vec4;                // C / Cin rows 4-element aligned: vector epilogue stores / loads
+  int noepi;               // experiment (PS_TC_NOEPI): skip the epilogue's stores (results invalid)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -194,6 +199,7 @@ __device__ __forceinline__ float epi_op(const Params &p, float r, float cin) {
 // the matching Cin load for alpha/beta).  fp8 operands: accumulator x 2^kab first.
 __device__ __forceinline__ void epi_chunk(const Params &p, float *stg, int lane, int64_t row0,
                                           int64_t col0, const uint32_t (&v)[32], int kab) {
+  if (p.noepi) return;
   float4 *srow = reinterpret_cast<float4 *>(stg + lane * EPI_STRIDE);
 #pragma unroll
   for (int q = 0; q < 8; q++)
@@ -357,13 +363,14 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       }
       umma_commit(tfull);         // accumulator complete
     }
-  } else {   // ------------------------- epilogue warps 2..5
+  } else {   // ------------------------- epilogue warps 2..9
     mbar_wait(tfull, 0);
     fence_after();
     const int kab = scale_exp2(p);
     const int q = warp & 3;                 // TMEM lane quarter this warp may access
     float *stg = epi_stage + (warp - 2) * 32 * EPI_STRIDE;
-    for (int cc = 0; cc < BN / EPI_COLS; cc++) {
+    const int half = (warp - 2) / 4;        // which half of the columns this warp drains
+    for (int cc = half * (BN / EPI_COLS / 2); cc < (half + 1) * (BN / EPI_COLS / 2); cc++) {
       if ((int64_t)n0 + cc * EPI_COLS >= p.N) break;
       uint32_t v[32];
       tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
@@ -389,13 +396,13 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 // c, c + #clusters, ... (SYRK: lower tiles skipped by every role alike).
 namespace tc2 {
 
-constexpr int BM = 256, BN = 256, STAGES = 6;
+constexpr int BM = 256, BN = 256, STAGES = 5;
 constexpr int HM = BM / 2, HN = BN / 2;          // per-CTA halves
 constexpr int A_BYTES = HM * tc::KB_BYTES;      // 16 KiB
 constexpr int B_BYTES = HN * tc::KB_BYTES;      // 16 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512 + tc::EPI_SMEM;
-constexpr int NTHREADS = 192;
+constexpr int NTHREADS = tc::NTHREADS;
 constexpr uint32_t TMEM_COLS = 512;             // 2 accumulators x 256 f32 columns
 constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;     // shared::cluster address of the leader's copy
 
@@ -512,7 +519,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
     }
     for (int a = 0; a < 2; a++) {
       mbar_init(&tfull[a], 1);
-      mbar_init(&tempty[a], 8);          // 4 epilogue warps x 2 CTAs
+      mbar_init(&tempty[a], 2 * tc::EPI_WARPS);   // every epilogue warp of both CTAs
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -590,7 +597,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
         j++;
       }
     }
-  } else {   // ------------------------- epilogue warps 2..5 (both CTAs)
+  } else {   // ------------------------- epilogue warps 2..9 (both CTAs)
     const int q = warp & 3;
     const int kab = scale_exp2(p);
     int64_t cursor = cluster;
@@ -602,7 +609,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
       fence_after();
       const int64_t row0 = (int64_t)m0 + rank * HM + q * 32;
       float *stg = epi_stage + (warp - 2) * 32 * EPI_STRIDE;
-      for (int cc = 0; cc < BN / EPI_COLS; cc++) {
+      const int half = (warp - 2) / 4;
+      for (int cc = half * (BN / EPI_COLS / 2); cc < (half + 1) * (BN / EPI_COLS / 2); cc++) {
         if ((int64_t)n0 + cc * EPI_COLS >= p.N) break;
         uint32_t v[32];
         tmem_ld32(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
@@ -706,7 +714,7 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   const uint32_t bfm = (g.B.type == PS_BF16 || g.B.type == PS_E5M2) ? 1u : 0u;
   Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, b_k ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
            (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, af, bfm,
-           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr, 0};
+           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr, 0, getenv("PS_TC_NOEPI") ? 1 : 0};
   {   // vector epilogue: rows of C (and Cin) start 16-byte (f32) / 8-byte (16-bit) aligned
     const int64_t cb = (int64_t)dtype_size(g.c_type);
     bool v4 = g.ldc % 4 == 0 && (uintptr_t)g.C % (4 * cb) == 0;
