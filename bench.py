@@ -554,9 +554,23 @@ def main():
             h2d += sum(x.numel() * 4 for x in hin if x is not None)
         d2h = sum(len(a["ids"]) * 24 for a in apps)      # one (sum e, max, count) record per config
 
+        copy = torch.cuda.Stream()
+
         def step_e2e():
+            # every app's H2D is issued up front on a copy stream (ps_app_load_host is
+            # asynchronous on its stream), so app k+1's inputs cross PCIe while app k's
+            # sweep runs; each sweep waits only for its own app's copy
+            go = torch.cuda.Event()
+            go.record(stream)
+            copy.wait_event(go)
+            ready = []
             for a, hin in zip(apps, host):
-                a["app"].load_host(hin)                               # H2D of the inputs
+                a["app"].load_host(hin, stream=copy)                 # H2D of the inputs
+                ev = torch.cuda.Event()
+                ev.record(copy)
+                ready.append(ev)
+            for a, ev in zip(apps, ready):
+                stream.wait_event(ev)
                 D.sharded_reference(a["app"], world, rank, refs=a["refs"])
                 arr, _ = a["app"].sweep_raw(a["ids"], args.toq)       # results read back (D2H)
                 if world > 1:
