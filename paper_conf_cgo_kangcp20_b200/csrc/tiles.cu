@@ -47,8 +47,14 @@ __global__ void __launch_bounds__(TTHREADS) tile_kernel(TileArgs a) {
   using RA = raw_t<SA>;
   constexpr int V = 16 / sizeof(RA);
   constexpr bool SAME = std::is_same<TC, TR>::value;
-  // rows per group: 16, or 8 when fp16 chunks (V = 8) meet an f64 compute type (registers)
-  constexpr int GR = (V == 8 && (sizeof(TC) == 8 || sizeof(TR) == 8)) ? 8 : 16;
+  // rows per group: 16, or 8 where 16 would take more than 128 registers (2 CTAs per
+  // SM instead of 1 keeps the same bytes in flight and fills all SMs; ptxas -v):
+  // 16-bit chunks (V = 8) with row dots or an f64 compute type, f32 chunks (V = 4)
+  // feeding f64 column sums or weighted (COL_DOT) f32 column sums without row dots
+  constexpr int GR = ((V == 8 && (RD || sizeof(TC) == 8 || sizeof(TR) == 8)) ||
+                      (V == 4 && !RD && (CM == COL_DOT || sizeof(TC) == 8)))
+                         ? 8
+                         : 16;
   __shared__ TR part[RD ? COLSUM_CHUNK : 1][TILE_SLABS + 1];
   __shared__ TC sw[CM == COL_DOT ? COLSUM_CHUNK : 1];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
