@@ -1,0 +1,268 @@
+// gemm_dmma.cu -- f64 contractions on the fp64 tensor-core MMA (DMMA) with
+// reading R3's summation order.
+//
+// R3: C_ij = sum_k A_ik B_kj is the fma chain acc <- fma(a_k, b_k, acc) from +0,
+// k ascending.  `mma.sync.m8n8k4.f64` computes D = A(8x4) B(4x8) + C; measured
+// on this B200 (tools/dmma_probe.cu, profiles/dmma_probe_r1.txt) its result is,
+// bit for bit, the chain d = fma(a3,b3, fma(a2,b2, fma(a1,b1, fma(a0,b0, c))))
+// -- C first, k ascending, one rounding per step -- over random, wide-exponent,
+// cancellation-heavy, subnormal and inf/NaN operands.  Chaining the MMAs over
+// k = 0, 4, 8, ... with the accumulator as C therefore reproduces R3 exactly
+// (the GPU parity tests check every f64 statement bit-exactly against the
+// oracle).  Operands are read in their stored precision and widened exactly to
+// f64 when staged in shared memory (R1); the epilogue is the SIMT kernel's.
+//
+// CTA tile 128 x 128, BK = 16, 8 warps of 64 x 32 (8 x 4 MMA tiles, 64 f64
+// accumulators per lane); register-prefetched, double-buffered shared tiles with
+// rows padded by 4 doubles so every fragment load (lane (r, q) reads element
+// (r, q) of an 8 x 4 block) is bank-conflict free.
+#include <cstdlib>
+#include <type_traits>
+
+#include "gemm_simt.cuh"
+
+namespace ps {
+namespace simt {
+
+// WGM x WGN warps; warp tile (BM / WGM) x (BN / WGN) = MI x NJ MMA tiles of 8 x 8
+template <int WGM, int WGN>
+struct DCfg {
+  static constexpr int BM = 128, BN = 128, BK = 16, THREADS = 32 * WGM * WGN, PAD = 4;
+  static constexpr int MI = BM / (8 * WGM), NJ = BN / (8 * WGN);
+  static constexpr int A_ELEMS = BM * (BK + PAD) > BK * (BM + PAD) ? BM * (BK + PAD) : BK * (BM + PAD);
+  static constexpr int B_ELEMS = BK * (BN + PAD);
+  static constexpr int SMEM = 2 * (A_ELEMS + B_ELEMS) * 8;
+};
+
+// Exact widening of stored f32 / f16 / bf16 bits to f64 with integer operations
+// (R1): cvt.f64.f32 / cvt.f64.f16 issue on the fp64 pipe the MMAs need, and cost
+// the mixed-storage statements ~20% (profiles/dmma_probe_r1.txt); the integer pipe
+// is otherwise idle here.  Normal numbers rebias the exponent and shift the fraction;
+// subnormals are renormalised (exact); inf keeps its sign; NaN stays NaN (quiet).
+__device__ __forceinline__ double f32bits_to_f64(uint32_t u) {
+  const uint32_t e = (u >> 23) & 0xffu, m = u & 0x7fffffu;
+  const uint64_t sign = (uint64_t)(u >> 31) << 63;
+  uint64_t r = sign | ((uint64_t)(e + 896u) << 52) | ((uint64_t)m << 29);
+  if (__builtin_expect(e - 1u >= 0xfeu, 0)) {
+    if (e == 0xffu) {
+      r = sign | (0x7ffull << 52) | ((uint64_t)m << 29) | (m ? (1ull << 51) : 0ull);
+    } else if (m == 0) {
+      r = sign;
+    } else {
+      const int p = 31 - __clz((int)m);   // leading bit: value = 1.f x 2^(p - 149)
+      r = sign | ((uint64_t)(p + 874) << 52) | (((uint64_t)m << (52 - p)) & 0xfffffffffffffull);
+    }
+  }
+  return __longlong_as_double((long long)r);
+}
+__device__ __forceinline__ double f16bits_to_f64(uint32_t h) {
+  const uint32_t e = (h >> 10) & 0x1fu, m = h & 0x3ffu;
+  const uint64_t sign = (uint64_t)((h >> 15) & 1u) << 63;
+  uint64_t r = sign | ((uint64_t)(e + 1008u) << 52) | ((uint64_t)m << 42);
+  if (__builtin_expect(e - 1u >= 0x1eu, 0)) {
+    if (e == 0x1fu) {
+      r = sign | (0x7ffull << 52) | ((uint64_t)m << 42) | (m ? (1ull << 51) : 0ull);
+    } else if (m == 0) {
+      r = sign;
+    } else {
+      const int p = 31 - __clz((int)m);   // value = 1.f x 2^(p - 24)
+      r = sign | ((uint64_t)(p + 999) << 52) | (((uint64_t)m << (52 - p)) & 0xfffffffffffffull);
+    }
+  }
+  return __longlong_as_double((long long)r);
+}
+template <class S> __device__ __forceinline__ double widen_i(raw_t<S> v) {
+  if constexpr (std::is_same<S, double>::value) return v;
+  else if constexpr (std::is_same<S, float>::value) return f32bits_to_f64(__float_as_uint(v));
+  else if constexpr (std::is_same<S, BF16>::value) return f32bits_to_f64((uint32_t)v << 16);
+  else return f32bits_to_f64(__float_as_uint(f16_to_f32(v)));   // cvt.f32.f16: exact, not the fp64 pipe
+}
+// E contiguous stored elements (16-byte aligned run), raw bits; widened at the
+// shared-memory store so the global loads stay in flight across the tile's MMAs
+template <class R, int E>
+__device__ __forceinline__ void load_run_raw(const R *p, R (&out)[E]) {
+  constexpr int BYTES = E * (int)sizeof(R);
+  if constexpr (BYTES >= 16) {
+    constexpr int PER = 16 / (int)sizeof(R);
+#pragma unroll
+    for (int q = 0; q < BYTES / 16; q++) {
+      union { uint4 u; R e[PER]; } t;
+      t.u = __ldg(reinterpret_cast<const uint4 *>(p) + q);
+#pragma unroll
+      for (int e = 0; e < PER; e++) out[q * PER + e] = t.e[e];
+    }
+  } else if constexpr (BYTES == 8) {
+    union { uint2 u; R e[E]; } t;
+    t.u = __ldg(reinterpret_cast<const uint2 *>(p));
+#pragma unroll
+    for (int e = 0; e < E; e++) out[e] = t.e[e];
+  } else {
+    static_assert(BYTES == 4, "4-byte run");
+    union { unsigned int u; R e[E]; } t;
+    t.u = __ldg(reinterpret_cast<const unsigned int *>(p));
+#pragma unroll
+    for (int e = 0; e < E; e++) out[e] = t.e[e];
+  }
+}
+
+__device__ __forceinline__ void dmma(double &d0, double &d1, double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+               : "+d"(d0), "+d"(d1)
+               : "d"(a), "d"(b));
+}
+
+template <class SA, class SB, bool AK, int WGM, int WGN>
+__global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
+    gemm_dmma_kernel(Params p, double alpha, double beta, double div) {
+  using DCfg = DCfg<WGM, WGN>;
+  constexpr int BM = DCfg::BM, BN = DCfg::BN, BK = DCfg::BK, PAD = DCfg::PAD, THREADS = DCfg::THREADS;
+  constexpr int MI = DCfg::MI, NJ = DCfg::NJ;
+  constexpr int LA = AK ? BK + PAD : BM + PAD;   // A row stride: [m][k] (AK) or [k][m]
+  constexpr int LB = BN + PAD;                   // B: [k][n]
+  constexpr int EA = BM * BK / THREADS, EB = BK * BN / THREADS;
+  extern __shared__ __align__(16) unsigned char smem_dyn[];
+  double *As0 = reinterpret_cast<double *>(smem_dyn);
+  double *Bs0 = As0 + 2 * DCfg::A_ELEMS;
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int r = lane >> 2, q = lane & 3;
+  const int wm = (warp / WGN) * (BM / WGM), wn = (warp % WGN) * (BN / WGN);
+  const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+  if (p.upper_only && m0 + p.row_off >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
+
+  const int a_m = AK ? tid / (BK / EA) : (tid % (BM / EA)) * EA;
+  const int a_k = AK ? (tid % (BK / EA)) * EA : tid / (BM / EA);
+  const int b_k = tid / (BN / EB), b_n = (tid % (BN / EB)) * EB;
+  const raw_t<SA> *Ap = (const raw_t<SA> *)p.A;
+  const raw_t<SB> *Bp = (const raw_t<SB> *)p.B;
+  const bool m_full = m0 + BM <= p.M, n_full = n0 + BN <= p.N;
+
+  raw_t<SA> ra[EA];   // raw stored bits (zero bits = +0 for every storage type)
+  raw_t<SB> rb[EB];
+  auto load_tiles = [&](int64_t k0) {
+    const bool k_full = k0 + BK <= p.K;
+    if (p.a_vec && m_full && k_full) {
+      load_run_raw<raw_t<SA>, EA>(Ap + (m0 + a_m) * p.a_sr + (k0 + a_k) * p.a_sc, ra);
+    } else {
+#pragma unroll
+      for (int e = 0; e < EA; e++) {
+        const int64_t gm = m0 + a_m + (AK ? 0 : e), gk = k0 + a_k + (AK ? e : 0);
+        ra[e] = (gm < p.M && gk < p.K) ? Ap[gm * p.a_sr + gk * p.a_sc] : raw_t<SA>(0);
+      }
+    }
+    if (p.b_vec && n_full && k_full) {
+      load_run_raw<raw_t<SB>, EB>(Bp + (k0 + b_k) * p.b_sr + n0 + b_n, rb);
+    } else {
+#pragma unroll
+      for (int e = 0; e < EB; e++) {
+        const int64_t gk = k0 + b_k, gn = n0 + b_n + e;
+        rb[e] = (gk < p.K && gn < p.N) ? Bp[gk * p.b_sr + gn] : raw_t<SB>(0);
+      }
+    }
+  };
+  auto store_tiles = [&](int buf) {
+    double *As = As0 + buf * DCfg::A_ELEMS, *Bs = Bs0 + buf * DCfg::B_ELEMS;
+    double2 *pa = reinterpret_cast<double2 *>(AK ? As + a_m * LA + a_k : As + a_k * LA + a_m);
+#pragma unroll
+    for (int e = 0; e < EA / 2; e++) pa[e] = make_double2(widen_i<SA>(ra[2 * e]), widen_i<SA>(ra[2 * e + 1]));
+    double2 *pb = reinterpret_cast<double2 *>(Bs + b_k * LB + b_n);
+#pragma unroll
+    for (int e = 0; e < EB / 2; e++) pb[e] = make_double2(widen_i<SB>(rb[2 * e]), widen_i<SB>(rb[2 * e + 1]));
+  };
+
+  double acc[MI][NJ][2];
+#pragma unroll
+  for (int i = 0; i < MI; i++)
+#pragma unroll
+    for (int j = 0; j < NJ; j++) acc[i][j][0] = acc[i][j][1] = 0.0;
+
+  const int64_t ktiles = (p.K + BK - 1) / BK;
+  load_tiles(0);
+  store_tiles(0);
+  __syncthreads();
+  int buf = 0;
+  for (int64_t kt = 0; kt < ktiles; kt++) {
+    const bool more = kt + 1 < ktiles;
+    if (more) load_tiles((kt + 1) * BK);
+    const double *As = As0 + buf * DCfg::A_ELEMS, *Bs = Bs0 + buf * DCfg::B_ELEMS;
+#pragma unroll
+    for (int kk = 0; kk < BK; kk += 4) {
+      double af[MI], bf[NJ];
+#pragma unroll
+      for (int i = 0; i < MI; i++)
+        af[i] = AK ? As[(wm + i * 8 + r) * LA + kk + q] : As[(kk + q) * LA + wm + i * 8 + r];
+#pragma unroll
+      for (int j = 0; j < NJ; j++) bf[j] = Bs[(kk + q) * LB + wn + j * 8 + r];
+#pragma unroll
+      for (int i = 0; i < MI; i++)
+#pragma unroll
+        for (int j = 0; j < NJ; j++) dmma(acc[i][j][0], acc[i][j][1], af[i], bf[j]);   // R3, k ascending
+    }
+    if (more) {
+      store_tiles(buf ^ 1);
+      __syncthreads();
+      buf ^= 1;
+    }
+  }
+
+  // epilogue (R3): plain / fma(alpha, acc, beta*Cin) / acc / div, then RNE store (R1)
+#pragma unroll
+  for (int i = 0; i < MI; i++) {
+    const int64_t gm = m0 + wm + i * 8 + r;
+    if (gm >= p.M) continue;
+#pragma unroll
+    for (int j = 0; j < NJ; j++) {
+#pragma unroll
+      for (int e = 0; e < 2; e++) {
+        const int64_t gn = n0 + wn + j * 8 + 2 * q + e;
+        if (gn >= p.N) continue;
+        double v = acc[i][j][e];
+        const int64_t idx = gm * p.ldc + gn;
+        if (p.epi == EPI_AXPBY) v = fma(alpha, v, beta * load_elem<double>(p.Cin, p.tcin, idx));
+        else if (p.epi == EPI_DIV) v = v / div;
+        store_elem<double>(p.C, p.tc, idx, v);
+      }
+    }
+  }
+}
+
+template <class SA, class SB, int WGM, int WGN>
+static ps_status launch_dmma(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
+  using C = DCfg<WGM, WGN>;
+  constexpr int SM = C::SMEM;
+  static bool attr = false;
+  if (!attr) {
+    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, true, WGM, WGN>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
+    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, false, WGM, WGN>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
+    attr = true;
+  }
+  dim3 grid((unsigned)((p.N + C::BN - 1) / C::BN), (unsigned)((p.M + C::BM - 1) / C::BM));
+  if (ak) gemm_dmma_kernel<SA, SB, true, WGM, WGN><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
+  else gemm_dmma_kernel<SA, SB, false, WGM, WGN><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
+  PS_CHECK_LAUNCH("gemm_dmma_kernel");
+  return PS_OK;
+}
+
+// PS_DMMA_WARPS=8 selects the 8-warp (64 x 32 warp tile) variant, else 16 warps (32 x 32)
+static int dmma_warps() {
+  static const int v = [] { const char *e = getenv("PS_DMMA_WARPS"); return e && atoi(e) == 8 ? 8 : 16; }();
+  return v;
+}
+
+ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st) {
+  const Params p = make_params(g);
+  const bool ak = g.A.s_col == 1;
+  return dispatch_store(g.A.type, [&](auto sa) -> ps_status {
+    return dispatch_store(g.B.type, [&](auto sb) -> ps_status {
+      using SA = decltype(sa);
+      using SB = decltype(sb);
+      return dmma_warps() == 8 ? launch_dmma<SA, SB, 2, 4>(p, ak, g.alpha, g.beta, g.div, st)
+                               : launch_dmma<SA, SB, 4, 4>(p, ak, g.alpha, g.beta, g.div, st);
+    });
+  });
+}
+
+}  // namespace simt
+}  // namespace ps

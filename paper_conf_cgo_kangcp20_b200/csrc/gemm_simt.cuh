@@ -240,6 +240,8 @@ inline Params make_params(const GemmArgs &g) {
 
 ps_status gemm_simt_f32(const GemmArgs &g, cudaStream_t st);
 ps_status gemm_simt_f64(const GemmArgs &g, cudaStream_t st);
+// f64 on the fp64 tensor-core MMA, R3 order (gemm_dmma.cu)
+ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st);
 
 }  // namespace simt
 }  // namespace ps

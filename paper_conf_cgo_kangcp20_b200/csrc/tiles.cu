@@ -192,8 +192,18 @@ __global__ void __launch_bounds__(256) colsum_finalize_kernel(const T *__restric
                                                               T eps) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= cols) return;
+  // chunks in order; loads issued 8 at a time so the in-order chain does not wait
+  // on one L2 round trip per term
   T total = partial[j];
-  for (int64_t c = 1; c < nchunks; c++) total = total + partial[c * cols + j];   // chunks in order
+  int64_t c = 1;
+  for (; c + 8 <= nchunks; c += 8) {
+    T v[8];
+#pragma unroll
+    for (int u = 0; u < 8; u++) v[u] = partial[(c + u) * cols + j];
+#pragma unroll
+    for (int u = 0; u < 8; u++) total = total + v[u];
+  }
+  for (; c < nchunks; c++) total = total + partial[c * cols + j];
   if (FIN == FIN_MEAN) total = total / n;
   if (FIN == FIN_STDDEV) {
     total = sqrt(total / n);
@@ -209,8 +219,16 @@ __global__ void __launch_bounds__(256) rowdot_finalize_kernel(const T *__restric
                                                               int64_t rows, int64_t ntiles, int add) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= rows) return;
-  T total = qpart[i];
-  for (int64_t t = 1; t < ntiles; t++) total = total + qpart[t * rows + i];   // tiles in order
+  T total = qpart[i];   // tiles in order, loads batched as in colsum_finalize_kernel
+  int64_t t = 1;
+  for (; t + 8 <= ntiles; t += 8) {
+    T v[8];
+#pragma unroll
+    for (int u = 0; u < 8; u++) v[u] = qpart[(t + u) * rows + i];
+#pragma unroll
+    for (int u = 0; u < 8; u++) total = total + v[u];
+  }
+  for (; t < ntiles; t++) total = total + qpart[t * rows + i];
   if (add) total = Ld<SO, T>::get(out, (size_t)i) + total;                   // MVT: x1 + A y1
   St<SO, T>::put(out, (size_t)i, total);
 }
