@@ -174,8 +174,10 @@ def _contractions(kind, d):
 def contraction_roofline(apps, last):
     """a3 of contraction workloads: frac = sum of ideal statement times (flops / the
     peak of the pipe the statement runs on) / sum of measured kernel times.  Peaks:
-    tensor = MEASURED_PEAKS bf16 burst (fp16 has the same dense rate); FFMA / DFMA
-    derived from unit counts (128 / 64 per SM per clock) x 148 SMs x 1965 MHz."""
+    tensor = MEASURED_PEAKS bf16 burst (fp16 has the same dense rate); FFMA and f64
+    derived from unit counts (128 / 64 FMA per SM per clock) x 148 SMs x 1965 MHz
+    (f64 statements run on the fp64 tensor-core MMA, DMMA: measured 37.0 TFLOP/s on a
+    pure-MMA loop, profiles/dmma_probe_r1.txt, so the derived 37.2 is the ceiling)."""
     _, tc_peak, _ = measured_peaks()
     peaks = {"tensor": tc_peak, 1: 148 * 128 * 2 * 1.965e9 / 1e12, 0: 148 * 64 * 2 * 1.965e9 / 1e12}
     ideal = meas = flops = 0.0
@@ -199,10 +201,10 @@ def contraction_roofline(apps, last):
     if meas <= 0:
         return None
     return {"bound": "tensor+fma", "achieved": round(flops / meas / 1e12, 2), "unit": "TFLOP/s",
-            "peak": {"tensor": tc_peak, "ffma": round(peaks[1], 1), "dfma": round(peaks[0], 1)},
+            "peak": {"tensor": tc_peak, "ffma": round(peaks[1], 1), "f64_dmma": round(peaks[0], 1)},
             "frac": round(ideal / meas, 4), "traffic": None,
             "peak_source": "tensor: MEASURED_PEAKS.json bf16_tflops (burst); FMA pipes derived",
-            "kernel": "a3 contraction statements (gemm_tc_kernel / gemm_simt_kernel)",
+            "kernel": "a3 contraction statements (gemm_tc2_kernel fp16/bf16/fp8, gemm_dmma_kernel f64, gemm_simt_kernel f32)",
             "statements_by_path": paths}
 
 

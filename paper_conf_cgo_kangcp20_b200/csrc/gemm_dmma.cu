@@ -25,13 +25,13 @@ namespace ps {
 namespace simt {
 
 // WGM x WGN warps; warp tile (BM / WGM) x (BN / WGN) = MI x NJ MMA tiles of 8 x 8
-template <int WGM, int WGN>
+template <int WGM, int WGN, int BK_ = 16, int STAGES_ = 4>
 struct DCfg {
-  static constexpr int BM = 128, BN = 128, BK = 16, THREADS = 32 * WGM * WGN, PAD = 4;
-  static constexpr int MI = BM / (8 * WGM), NJ = BN / (8 * WGN);
+  static constexpr int BM = 128, BN = 128, BK = BK_, THREADS = 32 * WGM * WGN, PAD = 4;
+  static constexpr int MI = BM / (8 * WGM), NJ = BN / (8 * WGN), STAGES = STAGES_;
   static constexpr int A_ELEMS = BM * (BK + PAD) > BK * (BM + PAD) ? BM * (BK + PAD) : BK * (BM + PAD);
   static constexpr int B_ELEMS = BK * (BN + PAD);
-  static constexpr int SMEM = 2 * (A_ELEMS + B_ELEMS) * 8;
+  static constexpr int SMEM = STAGES * (A_ELEMS + B_ELEMS) * 8;
 };
 
 // Exact widening of stored f32 / f16 / bf16 bits to f64 with integer operations
@@ -111,18 +111,36 @@ __device__ __forceinline__ void dmma(double &d0, double &d1, double a, double b)
                : "d"(a), "d"(b));
 }
 
-template <class SA, class SB, bool AK, int WGM, int WGN>
-__global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem));
+}
+// 8-byte copy, zero-filled when !valid (edge tiles and unaligned rows of f64 operands)
+__device__ __forceinline__ void cp_async8z(void *smem, const void *gmem, bool valid) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(gmem), "r"(valid ? 8 : 0));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N> __device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
+}
+
+template <class SA, class SB, bool AK, int WGM, int WGN, int BK_, int ST_>
+__global__ void __launch_bounds__(DCfg<WGM, WGN, BK_, ST_>::THREADS, 1)
     gemm_dmma_kernel(Params p, double alpha, double beta, double div) {
-  using DCfg = DCfg<WGM, WGN>;
+  using DCfg = DCfg<WGM, WGN, BK_, ST_>;
   constexpr int BM = DCfg::BM, BN = DCfg::BN, BK = DCfg::BK, PAD = DCfg::PAD, THREADS = DCfg::THREADS;
-  constexpr int MI = DCfg::MI, NJ = DCfg::NJ;
+  constexpr int MI = DCfg::MI, NJ = DCfg::NJ, S = DCfg::STAGES;
   constexpr int LA = AK ? BK + PAD : BM + PAD;   // A row stride: [m][k] (AK) or [k][m]
   constexpr int LB = BN + PAD;                   // B: [k][n]
   constexpr int EA = BM * BK / THREADS, EB = BK * BN / THREADS;
+  // f64-stored operands travel by cp.async (16 B = 2 doubles; 8 B zero-filled on edge
+  // tiles and unaligned rows), no registers; the others by register staging with
+  // exact widening at the shared-memory store
+  constexpr bool CA = std::is_same<SA, double>::value, CB = std::is_same<SB, double>::value;
   extern __shared__ __align__(16) unsigned char smem_dyn[];
   double *As0 = reinterpret_cast<double *>(smem_dyn);
-  double *Bs0 = As0 + 2 * DCfg::A_ELEMS;
+  double *Bs0 = As0 + S * DCfg::A_ELEMS;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int r = lane >> 2, q = lane & 3;
@@ -136,12 +154,38 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
   const raw_t<SA> *Ap = (const raw_t<SA> *)p.A;
   const raw_t<SB> *Bp = (const raw_t<SB> *)p.B;
   const bool m_full = m0 + BM <= p.M, n_full = n0 + BN <= p.N;
+  const int64_t ktiles = (p.K + BK - 1) / BK;
 
   raw_t<SA> ra[EA];   // raw stored bits (zero bits = +0 for every storage type)
   raw_t<SB> rb[EB];
-  auto load_tiles = [&](int64_t k0) {
+  // issue tile kt into stage st: cp.async for f64 operands, loads into ra / rb for the
+  // others (the returned flags say which operands still need store_regs)
+  auto issue = [&](int64_t kt, int st, bool &reg_a, bool &reg_b) {
+    const int64_t k0 = kt * BK;
     const bool k_full = k0 + BK <= p.K;
-    if (p.a_vec && m_full && k_full) {
+    double *As = As0 + st * DCfg::A_ELEMS, *Bs = Bs0 + st * DCfg::B_ELEMS;
+    const bool fa = p.a_vec && m_full && k_full, fb = p.b_vec && n_full && k_full;
+    reg_a = !CA;
+    reg_b = !CB;
+    if constexpr (CA) {
+#pragma unroll
+      for (int e = 0; e < BM * BK / 2 / THREADS; e++) {
+        const int c = tid + e * THREADS;
+        const int row = AK ? c / (BK / 2) : (c % (BM / 2)) * 2;   // m of the chunk's first element
+        const int kr = AK ? (c % (BK / 2)) * 2 : c / (BM / 2);     // k of the chunk's first element
+        double *dst = AK ? As + row * LA + kr : As + kr * LA + row;
+        if (fa) {
+          cp_async16(dst, Ap + (m0 + row) * p.a_sr + (k0 + kr) * p.a_sc);
+        } else {
+#pragma unroll
+          for (int h = 0; h < 2; h++) {
+            const int64_t gm = m0 + row + (AK ? 0 : h), gk = k0 + kr + (AK ? h : 0);
+            const bool ok = gm < p.M && gk < p.K;
+            cp_async8z(dst + h, ok ? Ap + gm * p.a_sr + gk * p.a_sc : Ap, ok);
+          }
+        }
+      }
+    } else if (fa) {
       load_run_raw<raw_t<SA>, EA>(Ap + (m0 + a_m) * p.a_sr + (k0 + a_k) * p.a_sc, ra);
     } else {
 #pragma unroll
@@ -150,7 +194,24 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
         ra[e] = (gm < p.M && gk < p.K) ? Ap[gm * p.a_sr + gk * p.a_sc] : raw_t<SA>(0);
       }
     }
-    if (p.b_vec && n_full && k_full) {
+    if constexpr (CB) {
+#pragma unroll
+      for (int e = 0; e < BK * BN / 2 / THREADS; e++) {
+        const int c = tid + e * THREADS;
+        const int kr = c / (BN / 2), nc = (c % (BN / 2)) * 2;
+        double *dst = Bs + kr * LB + nc;
+        if (fb) {
+          cp_async16(dst, Bp + (k0 + kr) * p.b_sr + n0 + nc);
+        } else {
+#pragma unroll
+          for (int h = 0; h < 2; h++) {
+            const int64_t gk = k0 + kr, gn = n0 + nc + h;
+            const bool ok = gk < p.K && gn < p.N;
+            cp_async8z(dst + h, ok ? Bp + gk * p.b_sr + gn : Bp, ok);
+          }
+        }
+      }
+    } else if (fb) {
       load_run_raw<raw_t<SB>, EB>(Bp + (k0 + b_k) * p.b_sr + n0 + b_n, rb);
     } else {
 #pragma unroll
@@ -160,14 +221,18 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
       }
     }
   };
-  auto store_tiles = [&](int buf) {
-    double *As = As0 + buf * DCfg::A_ELEMS, *Bs = Bs0 + buf * DCfg::B_ELEMS;
-    double2 *pa = reinterpret_cast<double2 *>(AK ? As + a_m * LA + a_k : As + a_k * LA + a_m);
+  auto store_regs = [&](int st, bool reg_a, bool reg_b) {
+    double *As = As0 + st * DCfg::A_ELEMS, *Bs = Bs0 + st * DCfg::B_ELEMS;
+    if (reg_a) {
+      double2 *pa = reinterpret_cast<double2 *>(AK ? As + a_m * LA + a_k : As + a_k * LA + a_m);
 #pragma unroll
-    for (int e = 0; e < EA / 2; e++) pa[e] = make_double2(widen_i<SA>(ra[2 * e]), widen_i<SA>(ra[2 * e + 1]));
-    double2 *pb = reinterpret_cast<double2 *>(Bs + b_k * LB + b_n);
+      for (int e = 0; e < EA / 2; e++) pa[e] = make_double2(widen_i<SA>(ra[2 * e]), widen_i<SA>(ra[2 * e + 1]));
+    }
+    if (reg_b) {
+      double2 *pb = reinterpret_cast<double2 *>(Bs + b_k * LB + b_n);
 #pragma unroll
-    for (int e = 0; e < EB / 2; e++) pb[e] = make_double2(widen_i<SB>(rb[2 * e]), widen_i<SB>(rb[2 * e + 1]));
+      for (int e = 0; e < EB / 2; e++) pb[e] = make_double2(widen_i<SB>(rb[2 * e]), widen_i<SB>(rb[2 * e + 1]));
+    }
   };
 
   double acc[MI][NJ][2];
@@ -176,15 +241,25 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
 #pragma unroll
     for (int j = 0; j < NJ; j++) acc[i][j][0] = acc[i][j][1] = 0.0;
 
-  const int64_t ktiles = (p.K + BK - 1) / BK;
-  load_tiles(0);
-  store_tiles(0);
-  __syncthreads();
-  int buf = 0;
+  // prologue: tiles 0 .. S-2 (one cp.async group each, possibly empty)
+#pragma unroll
+  for (int s = 0; s < S - 1; s++) {
+    if (s < ktiles) {
+      bool ga, gb;
+      issue(s, s, ga, gb);
+      store_regs(s, ga, gb);
+    }
+    cp_async_commit();
+  }
   for (int64_t kt = 0; kt < ktiles; kt++) {
-    const bool more = kt + 1 < ktiles;
-    if (more) load_tiles((kt + 1) * BK);
-    const double *As = As0 + buf * DCfg::A_ELEMS, *Bs = Bs0 + buf * DCfg::B_ELEMS;
+    cp_async_wait<S - 2>();   // this thread's copies of tile kt have landed
+    __syncthreads();          // everyone's have; everyone is done with tile kt-1's stage
+    const int64_t nt = kt + S - 1;
+    bool ga = false, gb = false;
+    if (nt < ktiles) issue(nt, (int)(nt % S), ga, gb);   // into the stage tile kt-1 used
+    cp_async_commit();
+    const int st = (int)(kt % S);
+    const double *As = As0 + st * DCfg::A_ELEMS, *Bs = Bs0 + st * DCfg::B_ELEMS;
 #pragma unroll
     for (int kk = 0; kk < BK; kk += 4) {
       double af[MI], bf[NJ];
@@ -198,12 +273,9 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
 #pragma unroll
         for (int j = 0; j < NJ; j++) dmma(acc[i][j][0], acc[i][j][1], af[i], bf[j]);   // R3, k ascending
     }
-    if (more) {
-      store_tiles(buf ^ 1);
-      __syncthreads();
-      buf ^= 1;
-    }
+    if (nt < ktiles) store_regs((int)(nt % S), ga, gb);   // register-staged operands of tile nt
   }
+  cp_async_wait<0>();
 
   // epilogue (R3): plain / fma(alpha, acc, beta*Cin) / acc / div, then RNE store (R1)
 #pragma unroll
@@ -226,28 +298,29 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN>::THREADS, 1)
   }
 }
 
-template <class SA, class SB, int WGM, int WGN>
+template <class SA, class SB, int WGM, int WGN, int BK, int ST>
 static ps_status launch_dmma(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
-  using C = DCfg<WGM, WGN>;
+  using C = DCfg<WGM, WGN, BK, ST>;
   constexpr int SM = C::SMEM;
   static bool attr = false;
   if (!attr) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, true, WGM, WGN>,
+    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
-    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, false, WGM, WGN>,
+    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
     attr = true;
   }
   dim3 grid((unsigned)((p.N + C::BN - 1) / C::BN), (unsigned)((p.M + C::BM - 1) / C::BM));
-  if (ak) gemm_dmma_kernel<SA, SB, true, WGM, WGN><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
-  else gemm_dmma_kernel<SA, SB, false, WGM, WGN><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
+  if (ak) gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
+  else gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
   PS_CHECK_LAUNCH("gemm_dmma_kernel");
   return PS_OK;
 }
 
-// PS_DMMA_WARPS=8 selects the 8-warp (64 x 32 warp tile) variant, else 16 warps (32 x 32)
-static int dmma_warps() {
-  static const int v = [] { const char *e = getenv("PS_DMMA_WARPS"); return e && atoi(e) == 8 ? 8 : 16; }();
+// Variant (measurement switch PS_DMMA_VARIANT): 0 = 16 warps, BK 32, 3 stages (default);
+// 1 = 16 warps, BK 16, 4 stages; 2 = 8 warps (64 x 32 warp tiles), BK 16, 4 stages
+static int dmma_variant() {
+  static const int v = [] { const char *e = getenv("PS_DMMA_VARIANT"); return e ? atoi(e) : 0; }();
   return v;
 }
 
@@ -258,8 +331,11 @@ ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st) {
     return dispatch_store(g.B.type, [&](auto sb) -> ps_status {
       using SA = decltype(sa);
       using SB = decltype(sb);
-      return dmma_warps() == 8 ? launch_dmma<SA, SB, 2, 4>(p, ak, g.alpha, g.beta, g.div, st)
-                               : launch_dmma<SA, SB, 4, 4>(p, ak, g.alpha, g.beta, g.div, st);
+      switch (dmma_variant()) {
+        case 1: return launch_dmma<SA, SB, 4, 4, 16, 4>(p, ak, g.alpha, g.beta, g.div, st);
+        case 2: return launch_dmma<SA, SB, 2, 4, 16, 4>(p, ak, g.alpha, g.beta, g.div, st);
+        default: return launch_dmma<SA, SB, 4, 4, 32, 3>(p, ak, g.alpha, g.beta, g.div, st);
+      }
     });
   });
 }
