@@ -12,9 +12,11 @@
 // oracle).  Operands are read in their stored precision and widened exactly to
 // f64 when staged in shared memory (R1); the epilogue is the SIMT kernel's.
 //
-// CTA tile 128 x 128, BK = 16, 8 warps of 64 x 32 (8 x 4 MMA tiles, 64 f64
-// accumulators per lane); register-prefetched, double-buffered shared tiles with
-// rows padded by 4 doubles so every fragment load (lane (r, q) reads element
+// Default shape: CTA tile 128 x 64, 8 warps of 32 x 32 (4 x 4 MMA tiles, 32 f64
+// accumulators per lane), two CTAs per SM (one's barrier stalls are covered by the
+// other's MMAs), a 3-stage ring of BK = 16 tiles: cp.async for f64 operands,
+// register staging with exact integer widening for f32/f16/bf16 ones.  Shared
+// rows are padded by 4 doubles so every fragment load (lane (r, q) reads element
 // (r, q) of an 8 x 4 block) is bank-conflict free.
 #include <cstdlib>
 #include <type_traits>
@@ -25,9 +27,9 @@ namespace ps {
 namespace simt {
 
 // WGM x WGN warps; warp tile (BM / WGM) x (BN / WGN) = MI x NJ MMA tiles of 8 x 8
-template <int WGM, int WGN, int BK_ = 16, int STAGES_ = 4>
+template <int WGM, int WGN, int BK_ = 16, int STAGES_ = 4, int BN_ = 128, int MINB_ = 1>
 struct DCfg {
-  static constexpr int BM = 128, BN = 128, BK = BK_, THREADS = 32 * WGM * WGN, PAD = 4;
+  static constexpr int BM = 128, BN = BN_, BK = BK_, THREADS = 32 * WGM * WGN, PAD = 4, MINB = MINB_;
   static constexpr int MI = BM / (8 * WGM), NJ = BN / (8 * WGN), STAGES = STAGES_;
   static constexpr int A_ELEMS = BM * (BK + PAD) > BK * (BM + PAD) ? BM * (BK + PAD) : BK * (BM + PAD);
   static constexpr int B_ELEMS = BK * (BN + PAD);
@@ -77,58 +79,16 @@ template <class S> __device__ __forceinline__ double widen_i(raw_t<S> v) {
   else if constexpr (std::is_same<S, BF16>::value) return f32bits_to_f64((uint32_t)v << 16);
   else return f32bits_to_f64(__float_as_uint(f16_to_f32(v)));   // cvt.f32.f16: exact, not the fp64 pipe
 }
-// E contiguous stored elements (16-byte aligned run), raw bits; widened at the
-// shared-memory store so the global loads stay in flight across the tile's MMAs
-template <class R, int E>
-__device__ __forceinline__ void load_run_raw(const R *p, R (&out)[E]) {
-  constexpr int BYTES = E * (int)sizeof(R);
-  if constexpr (BYTES >= 16) {
-    constexpr int PER = 16 / (int)sizeof(R);
-#pragma unroll
-    for (int q = 0; q < BYTES / 16; q++) {
-      union { uint4 u; R e[PER]; } t;
-      t.u = __ldg(reinterpret_cast<const uint4 *>(p) + q);
-#pragma unroll
-      for (int e = 0; e < PER; e++) out[q * PER + e] = t.e[e];
-    }
-  } else if constexpr (BYTES == 8) {
-    union { uint2 u; R e[E]; } t;
-    t.u = __ldg(reinterpret_cast<const uint2 *>(p));
-#pragma unroll
-    for (int e = 0; e < E; e++) out[e] = t.e[e];
-  } else {
-    static_assert(BYTES == 4, "4-byte run");
-    union { unsigned int u; R e[E]; } t;
-    t.u = __ldg(reinterpret_cast<const unsigned int *>(p));
-#pragma unroll
-    for (int e = 0; e < E; e++) out[e] = t.e[e];
-  }
-}
-
 __device__ __forceinline__ void dmma(double &d0, double &d1, double a, double b) {
   asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
                : "+d"(d0), "+d"(d1)
                : "d"(a), "d"(b));
 }
 
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem));
-}
-// 8-byte copy, zero-filled when !valid (edge tiles and unaligned rows of f64 operands)
-__device__ __forceinline__ void cp_async8z(void *smem, const void *gmem, bool valid) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(gmem), "r"(valid ? 8 : 0));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-template <int N> __device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
-}
-
-template <class SA, class SB, bool AK, int WGM, int WGN, int BK_, int ST_>
-__global__ void __launch_bounds__(DCfg<WGM, WGN, BK_, ST_>::THREADS, 1)
+template <class SA, class SB, bool AK, int WGM, int WGN, int BK_, int ST_, int BN_, int MB_>
+__global__ void __launch_bounds__(DCfg<WGM, WGN, BK_, ST_, BN_, MB_>::THREADS, MB_)
     gemm_dmma_kernel(Params p, double alpha, double beta, double div) {
-  using DCfg = DCfg<WGM, WGN, BK_, ST_>;
+  using DCfg = DCfg<WGM, WGN, BK_, ST_, BN_, MB_>;
   constexpr int BM = DCfg::BM, BN = DCfg::BN, BK = DCfg::BK, PAD = DCfg::PAD, THREADS = DCfg::THREADS;
   constexpr int MI = DCfg::MI, NJ = DCfg::NJ, S = DCfg::STAGES;
   constexpr int LA = AK ? BK + PAD : BM + PAD;   // A row stride: [m][k] (AK) or [k][m]
@@ -298,27 +258,32 @@ __global__ void __launch_bounds__(DCfg<WGM, WGN, BK_, ST_>::THREADS, 1)
   }
 }
 
-template <class SA, class SB, int WGM, int WGN, int BK, int ST>
+template <class SA, class SB, int WGM, int WGN, int BK, int ST, int BN = 128, int MB = 1>
 static ps_status launch_dmma(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
-  using C = DCfg<WGM, WGN, BK, ST>;
+  using C = DCfg<WGM, WGN, BK, ST, BN, MB>;
   constexpr int SM = C::SMEM;
   static bool attr = false;
   if (!attr) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST>,
+    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST, BN, MB>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
-    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST>,
+    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST, BN, MB>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
     attr = true;
   }
   dim3 grid((unsigned)((p.N + C::BN - 1) / C::BN), (unsigned)((p.M + C::BM - 1) / C::BM));
-  if (ak) gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
-  else gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
+  if (ak) gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST, BN, MB><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
+  else gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST, BN, MB><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
   PS_CHECK_LAUNCH("gemm_dmma_kernel");
   return PS_OK;
 }
 
-// Variant (measurement switch PS_DMMA_VARIANT): 0 = 16 warps, BK 32, 3 stages (default);
-// 1 = 16 warps, BK 16, 4 stages; 2 = 8 warps (64 x 32 warp tiles), BK 16, 4 stages
+// Variant (measurement switch PS_DMMA_VARIANT; f64 GEMM at 8192^3, profiles/dmma_probe_r1.txt):
+//   0 (default) 128 x 64 CTA tiles of 8 warps (32 x 32 warp tiles), two CTAs per SM,
+//     3 stages of BK 16: 34.2 TFLOP/s
+//   1 128 x 128 tiles of 16 warps, one CTA per SM, 4 stages of BK 16: 29.9
+//   2 128 x 128 tiles of 8 warps (64 x 32 warp tiles), 4 stages of BK 16
+//   3 128 x 128 tiles of 16 warps, 3 stages of BK 32: 31.5
+//   4 128 x 64 tiles, two CTAs per SM, 2 stages of BK 32: 32.3
 static int dmma_variant() {
   static const int v = [] { const char *e = getenv("PS_DMMA_VARIANT"); return e ? atoi(e) : 0; }();
   return v;
@@ -334,7 +299,9 @@ ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st) {
       switch (dmma_variant()) {
         case 1: return launch_dmma<SA, SB, 4, 4, 16, 4>(p, ak, g.alpha, g.beta, g.div, st);
         case 2: return launch_dmma<SA, SB, 2, 4, 16, 4>(p, ak, g.alpha, g.beta, g.div, st);
-        default: return launch_dmma<SA, SB, 4, 4, 32, 3>(p, ak, g.alpha, g.beta, g.div, st);
+        case 3: return launch_dmma<SA, SB, 4, 4, 32, 3>(p, ak, g.alpha, g.beta, g.div, st);
+        case 4: return launch_dmma<SA, SB, 4, 2, 32, 2, 64, 2>(p, ak, g.alpha, g.beta, g.div, st);
+        default: return launch_dmma<SA, SB, 4, 2, 16, 3, 64, 2>(p, ak, g.alpha, g.beta, g.div, st);
       }
     });
   });

@@ -98,6 +98,53 @@ __device__ __forceinline__ void load_run(const raw_t<S> *p, T (&out)[E]) {
   }
 }
 
+// ---- cp.async and raw-run helpers (gemm_dmma.cu, gemm_ffma.cu)
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem));
+}
+// 4- / 8-byte copies, zero-filled when !valid (edge tiles and unaligned rows of f64 operands)
+__device__ __forceinline__ void cp_async8z(void *smem, const void *gmem, bool valid) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(sa), "l"(gmem), "r"(valid ? 8 : 0));
+}
+__device__ __forceinline__ void cp_async4z(void *smem, const void *gmem, bool valid) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(sa), "l"(gmem), "r"(valid ? 4 : 0));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N> __device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
+}
+
+// E contiguous stored elements (16-byte aligned run), raw bits; widened at the
+// shared-memory store so the global loads stay in flight across the tile's MMAs
+template <class R, int E>
+__device__ __forceinline__ void load_run_raw(const R *p, R (&out)[E]) {
+  constexpr int BYTES = E * (int)sizeof(R);
+  if constexpr (BYTES >= 16) {
+    constexpr int PER = 16 / (int)sizeof(R);
+#pragma unroll
+    for (int q = 0; q < BYTES / 16; q++) {
+      union { uint4 u; R e[PER]; } t;
+      t.u = __ldg(reinterpret_cast<const uint4 *>(p) + q);
+#pragma unroll
+      for (int e = 0; e < PER; e++) out[q * PER + e] = t.e[e];
+    }
+  } else if constexpr (BYTES == 8) {
+    union { uint2 u; R e[E]; } t;
+    t.u = __ldg(reinterpret_cast<const uint2 *>(p));
+#pragma unroll
+    for (int e = 0; e < E; e++) out[e] = t.e[e];
+  } else {
+    static_assert(BYTES == 4, "4-byte run");
+    union { unsigned int u; R e[E]; } t;
+    t.u = __ldg(reinterpret_cast<const unsigned int *>(p));
+#pragma unroll
+    for (int e = 0; e < E; e++) out[e] = t.e[e];
+  }
+}
+
 template <class T, class SA, class SB, bool AK>
 __global__ void __launch_bounds__(Cfg<T>::THREADS, 1) gemm_kernel(Params p, T alpha, T beta, T div) {
   constexpr int BM = Cfg<T>::BM, BN = Cfg<T>::BN, BK = Cfg<T>::BK;
@@ -241,6 +288,8 @@ inline Params make_params(const GemmArgs &g) {
 ps_status gemm_simt_f32(const GemmArgs &g, cudaStream_t st);
 ps_status gemm_simt_f64(const GemmArgs &g, cudaStream_t st);
 // f64 on the fp64 tensor-core MMA, R3 order (gemm_dmma.cu)
+// f32 FFMA chains, two CTAs per SM, cp.async ring (gemm_ffma.cu)
+ps_status gemm_ffma_f32(const GemmArgs &g, cudaStream_t st);
 ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st);
 
 }  // namespace simt
