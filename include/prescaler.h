@@ -146,7 +146,10 @@ PS_API ps_status ps_app_destroy(ps_app *app);
 PS_API int ps_app_num_objects(const ps_app *app);            /* -1 if app == NULL */
 PS_API ps_status ps_app_object_info(const ps_app *app, int m, ps_object_info *out);
 /* flags: PS_FLAG_NO_TENSOR_CORES forces the SIMT contraction path for fp16   */
-/* operands (bit-exact with R3) instead of tcgen05 (tolerance R6).            */
+/* operands (bit-exact with R3) instead of tcgen05 (tolerance R6).  It does   */
+/* not concern f64 statements: they always run on the fp64 MMA (mma.sync     */
+/* .f64), whose chained result is R3's fma chain bit for bit (measured,       */
+/* profiles/dmma_probe_r1.txt).                          */
 /* PS_FLAG_BF16 extends the configuration alphabet to {f64, f32, f16, bf16}:  */
 /* precision vectors may hold PS_BF16 and ids run over 4^M (radix 4, object 0 */
 /* least significant); without it the space is the paper's 3^M.               */

@@ -1,5 +1,5 @@
 """f64 contractions: the DMMA kernel (gemm_dmma.cu, the default) and the DFMA
-kernel (gemm_simt.cuh, PS_F64_DFMA=1) are both bit-exact with reading R3's fma
+kernel (gemm_simt.cuh, PS_F64_DFMA=1) are both bit-exact (and so are both f32 kernels) with reading R3's fma
 chain.  The DMMA kernel relies on mma.sync .f64 computing fma(a3,b3, ... fma(a0,b0,c))
 (measured: profiles/dmma_probe_r1.txt); these inputs are built so that any other
 summation order or a fused dot product would change results: wide exponent
@@ -66,10 +66,12 @@ def test_f64_statements_bit_exact_adversarial(torch, kind, dims, sc):
             check_config(torch, app, kind, dims, ins, oref, prec, sc)
 
 
-def test_dfma_kernel_bit_exact():
-    """The SIMT DFMA kernel behind PS_F64_DFMA=1 (kept for measurement) stays R3-exact:
-    the contraction apps' exhaustive SIMT parity cases in a child process."""
-    env = dict(os.environ, PS_F64_DFMA="1")
+@pytest.mark.parametrize("switch", ["PS_F64_DFMA", "PS_F32_SIMT_OLD"])
+def test_previous_kernels_bit_exact(switch):
+    """The kernels kept behind measurement switches (the DFMA f64 kernel, PS_F64_DFMA=1;
+    the previous FFMA kernel, PS_F32_SIMT_OLD=1) stay R3-exact: the contraction apps'
+    exhaustive SIMT parity cases in a child process."""
+    env = dict(os.environ, **{switch: "1"})
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-p", "no:cacheprovider", "-m", "gpu",
                         os.path.join(ROOT, "tests", "test_gpu_apps.py"),
                         "-k", "gemm or 2mm or 3mm or corr or covar or syrk or syr2k"],
