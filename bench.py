@@ -39,7 +39,7 @@ WORKLOADS = {
     # BASELINE.json configs[0]
     "gemm64": [("gemm", [64])],
     # BASELINE.json configs[3] / configs[4] (3MM's 2187-config space at N=8192 is a
-    # separate workload: one step is minutes of fp64 DFMA on one GPU)
+    # separate workload: one step is minutes of fp64 MMA on one GPU)
     "contract": [("2mm", [8192])],
     "contract3mm": [("3mm", [8192])],
     "corr": [("corr", [8192, 8192]), ("covar", [8192, 8192])],
