@@ -10,11 +10,16 @@ Default workload = BASELINE.json configs[2]: ATAX, BICG, GESUMMV at N=16384
 TOQ 0.9.  configs[1] (the conversion sweep) is a single row (a2) of the path,
 so it is reported as the secondary `conversion_gbs` key, not as the step.
 
-Multi-GPU (torchrun, one process per GPU): the config space of every app is
-partitioned across ranks (deterministic LPT over a cost model); each rank
-evaluates its share; one NCCL all_gather of the 64-byte result records per app
-per step.  Timing: barrier + synchronize on both sides of exactly --steps
-steps, CUDA events on the launching stream, max over ranks.
+Multi-GPU (one process per GPU): ``--gpus N`` without a torchrun environment
+re-executes this script under ``torch.distributed.run`` with N ranks (127.0.0.1
+rendezvous); under torchrun (the driver's launch) the ranks come from the env.
+The config space of every app is partitioned across ranks (deterministic LPT
+over a cost model); each rank evaluates its share; one NCCL all_gather of the
+64-byte result records per app per step; the contraction apps' fp64 reference
+is row-sharded and all-gathered.  Timing: setup and warm-up first, then barrier
++ synchronize on both sides of exactly --steps steps, CUDA events on the
+launching stream, max over ranks.  ``--backend gloo --fake`` is a CPU dry run of
+the same orchestration (fake result records, no GPU) used by the CPU tests.
 
 --impl reference times the CPU oracle (oracle/, the plain C definition) as it
 stands on the host cores, on a bounded sample of the same workload.
@@ -61,6 +66,13 @@ CPU_SAMPLE = {"matvec": (8192, 2), "gemm64": (None, 0), "contract": (384, 3), "c
               "syr2k": (384, 3), "stencil3d": (128, 3), "fdtd": (None, 0)}
 # per-dimension sample overrides (the exponent then counts the scaled dimensions)
 CPU_SAMPLE_DIMS = {"fdtd": [50, 1024, 1024]}
+# GPU counts BASELINE.json names per workload (configs[2]: 1 and 2; [3]: 4; [4]: 8)
+BASELINE_GPUS = {"matvec": [1, 2], "contract": [4], "contract3mm": [4], "corr": [8], "gemm64": [1]}
+# BASELINE.md "paper context line": the paper's headline, other hardware -- context only
+PAPER_CONTEXT = {
+    "speedup": 1.33, "metric": "average whole-program speedup over the original precision at TOQ 0.9",
+    "hardware": "Titan Xp + Xeon E5-2640v4, PCIe 3.0 x16, OpenCL 1.2", "workload": "14 PolyBench apps",
+    "cite": "PAPER.md:388 (also 1.38x V100, 1.47x RTX 2080 Ti)", "context_only": True}
 
 
 def log(*a):
@@ -248,11 +260,20 @@ def stencil_roofline(apps, last, hbm):
             "ideal_time_share": {k2: round(v / ideal, 4) for k2, v in bound_t.items()}}
 
 
-def convert_bytes(objects, prec):
+CNAME = {0: "f32->f64", 1: "f32->f32 copy", 2: "f32->f16", 3: "f32->bf16"}
+
+
+def convert_bytes(objects, prec, by_dir=None):
+    """Algorithmic bytes of one configuration's a2 conversions (orig f32 -> c(m) for every
+    object read before written; inout objects are copied even at f32); by_dir (dict)
+    receives the bytes per direction."""
     b = 0
     for o, p in zip(objects, prec):
         if o["role"] in (0, 2) and (p != 1 or o["role"] == 2):
-            b += o["n"] * (4 + SIZE[p])
+            x = o["n"] * (4 + SIZE[p])
+            b += x
+            if by_dir is not None:
+                by_dir[CNAME[p]] = by_dir.get(CNAME[p], 0) + x
     return b
 
 
@@ -405,19 +426,34 @@ def whole_program(torch, B, apps, args):
 
 
 # ------------------------------------------------------------ conversion
+CONV_DIRECTIONS = [(1, 2, "f32->f16"), (2, 1, "f16->f32"), (0, 2, "f64->f16"), (0, 1, "f64->f32"),
+                   (1, 0, "f32->f64"), (1, 3, "f32->bf16")]
+CSIZE = {0: 8, 1: 4, 2: 2, 3: 2}
+
+
+def random_bits(torch, nbytes):
+    """Uniform random bit patterns (every class: normals, subnormals, +-inf, NaNs), so the
+    measured speed is value-independent."""
+    g = torch.Generator(device="cuda")
+    g.manual_seed(20200222)
+    n = nbytes // 4
+    return torch.randint(-2 ** 31, 2 ** 31 - 1, (n,), dtype=torch.int32, device="cuda", generator=g)
+
+
 def conversion_sweep(torch, B, flush, reps=20, sizes=None):
-    """BASELINE configs[1] / SURVEY §8(d)-2 row 2: source sizes 2^20 .. 2^32 bytes, four
-    directions, L2 flushed before every rep, median of `reps` CUDA-event timings.
-    Algorithmic GB/s = n (s_src + s_dst) / t."""
+    """BASELINE configs[1] / SURVEY §8(d)-2 row 2: source sizes 2^20 .. 2^32 bytes, the four
+    BASELINE directions plus f32->f64 (the a2 direction of every f64 configuration) and
+    f32->bf16, random bit patterns, L2 flushed before every rep, median of `reps` CUDA-event
+    timings.  Algorithmic GB/s = n (s_src + s_dst) / t."""
     sizes = sizes or [1 << k for k in range(20, 33)]
     out = {}
-    TD = {0: torch.float64, 1: torch.float32, 2: torch.float16}
-    for st, dt, name in [(1, 2, "f32->f16"), (2, 1, "f16->f32"), (0, 2, "f64->f16"),
-                         (0, 1, "f64->f32")]:
+    TD = {0: torch.float64, 1: torch.float32, 2: torch.float16, 3: torch.bfloat16}
+    bits = random_bits(torch, max(sizes))
+    for st, dt, name in CONV_DIRECTIONS:
         row = {}
         for nbytes in sizes:
-            n = nbytes // SIZE[st]
-            src = torch.zeros(n, dtype=TD[st], device="cuda")
+            n = nbytes // CSIZE[st]
+            src = bits[:nbytes // 4].view(TD[st])[:n]
             dst = torch.empty(n, dtype=TD[dt], device="cuda")
             for _ in range(3):
                 B.ps_convert(src, st, dst, dt)
@@ -431,10 +467,103 @@ def conversion_sweep(torch, B, flush, reps=20, sizes=None):
                 torch.cuda.synchronize()
                 ts.append(e0.elapsed_time(e1))
             t = float(np.median(ts))
-            row[nbytes] = round(n * (SIZE[st] + SIZE[dt]) / (t * 1e-3) / 1e9, 1)
-            del src, dst
+            row[nbytes] = round(n * (CSIZE[st] + CSIZE[dt]) / (t * 1e-3) / 1e9, 1)
+            del dst
         out[name] = row
+    del bits
     return out
+
+
+# ------------------------------------------------------------- launching
+def _free_port() -> int:
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def spawn_ranks(n: int) -> int:
+    """`bench.py --gpus N` outside torchrun: re-run this script as N ranks (one
+    process per GPU) under torch.distributed.run; rank 0 prints the line."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(n),
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
+           os.path.abspath(__file__)] + sys.argv[1:]
+    log("spawning %d ranks: %s" % (n, " ".join(cmd)))
+    return subprocess.call(cmd)
+
+
+def fake_records(ids, costs):
+    """--fake: deterministic stand-in for ps_sweep records (CPU dry run, no GPU):
+    total_ms = the cost model's prediction, quality from the id."""
+    import paper_conf_cgo_kangcp20_b200.binding as B
+    rec = np.zeros(len(ids), dtype=B.RESULT_DTYPE)
+    rec["config_id"] = np.asarray(ids, dtype=np.uint64)
+    rec["total_ms"] = np.asarray(costs, dtype=np.float32) * 1e3
+    rec["quality"] = 1.0 - (np.asarray(ids, dtype=np.uint64) * np.uint64(2654435761) % np.uint64(1000)) / 5e3
+    rec["pass"] = (rec["quality"] >= 0.9).astype(np.int32)
+    return rec
+
+
+def run_fake(args, rank, world):
+    """The multi-rank orchestration of the real run -- partition, per-rank sweep,
+    record gather, best config, max-over-ranks timing, one line from rank 0 --
+    with fake records and the gloo backend, so it runs (and is tested) on CPU."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_cgo_kangcp20_b200 import binding as B
+    from paper_conf_cgo_kangcp20_b200 import dist as D
+    if world > 1:
+        dist.init_process_group(args.backend)
+    apps = []
+    for kind, dims in WORKLOADS[args.workload]:
+        app = B.App(kind, dims)          # host metadata only
+        ids = list(range(app.space))
+        mine = D.partition_configs(kind, dims, app.objects, ids, world, rank) if world > 1 else ids
+        costs = [D.config_cost(kind, dims, app.objects, c) for c in mine]
+        apps.append(dict(kind=kind, ids=mine, costs=costs, space=app.space))
+    total = sum(a["space"] for a in apps)
+
+    def step():
+        best = {}
+        for a in apps:
+            arr = fake_records(a["ids"], a["costs"])
+            if world > 1:
+                arr = D.gather_results(arr)
+            assert len(arr) == a["space"]
+            best[a["kind"]] = int(arr["config_id"][D.best_index(arr)]) if D.best_index(arr) >= 0 else -1
+        return best
+
+    for _ in range(args.warmup):
+        step()
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        best = step()
+    el = time.perf_counter() - t0
+    el_t = torch.tensor([el], dtype=torch.float64)
+    counts = torch.tensor([sum(len(a["ids"]) for a in apps)], dtype=torch.int64)
+    allc = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+    if world > 1:
+        dist.all_reduce(el_t, op=dist.ReduceOp.MAX)
+        dist.all_gather(allc, counts)
+    else:
+        allc = [counts]
+    if rank == 0:
+        line = {"metric": "configs evaluated/s", "value": total * args.steps / el_t.item(),
+                "unit": "configs/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": el_t.item() / args.steps * 1e3, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "none (fake records)",
+                "data": "FAKE: CPU dry run of the multi-rank orchestration, no GPU, not a measurement",
+                "fake": True, "backend": args.backend,
+                "config": {"workload": args.workload, "configs_per_step": total,
+                           "configs_per_rank": [int(c.item()) for c in allc], "best_config": best}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
 
 
 # ------------------------------------------------------------------- main
@@ -447,6 +576,9 @@ def main():
     ap.add_argument("--workload", default="matvec", choices=sorted(WORKLOADS))
     ap.add_argument("--input-set", default="default", choices=["default", "random", "image"])
     ap.add_argument("--toq", type=float, default=0.9)
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"])
+    ap.add_argument("--fake", action="store_true",
+                    help="CPU dry run of the multi-rank orchestration (fake records; needs --backend gloo)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-conversion", action="store_true")
@@ -460,11 +592,19 @@ def main():
     elif args.warmup < 3:
         log("warmup raised to 3 (timing rule)")
         args.warmup = 3
+    if args.fake and args.backend != "gloo":
+        ap.error("--fake runs on CPU: use --backend gloo")
 
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        return spawn_ranks(args.gpus)
     rank, world = int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    if world != args.gpus and args.impl == "ours":
+        log("note: --gpus %d but WORLD_SIZE %d; the run uses %d rank(s)" % (args.gpus, world, world))
     if args.impl == "reference":
         return run_reference_arm(args, rank, world)
+    if args.fake:
+        return run_fake(args, rank, world)
 
     import torch
     import torch.distributed as dist
@@ -476,7 +616,7 @@ def main():
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.init_process_group(args.backend, device_id=torch.device("cuda", local))
     if rank == 0:
         build_mod.build()
     if world > 1:
@@ -543,6 +683,12 @@ def main():
         dist.all_reduce(lt, op=dist.ReduceOp.SUM)
         launches = int(lt.item())
     value = total_configs * args.steps / (el_ms * 1e-3)
+    per_rank = [sum(len(a["ids"]) for a in apps)]
+    if world > 1:
+        c = torch.tensor([per_rank[0]], dtype=torch.int64, device="cuda")
+        allc = torch.zeros(world, dtype=torch.int64, device="cuda")
+        dist.all_gather_into_tensor(allc, c)
+        per_rank = [int(x) for x in allc.cpu().tolist()]
 
     # ------------------------------------------------- e2e through host buffers
     e2e = None
@@ -607,6 +753,7 @@ def main():
     hbm, _, peak_src = measured_peaks()
     phase = {"convert": 0.0, "kernel": 0.0, "backconv": 0.0, "quality": 0.0}
     kb = kt = cb = ct = 0.0
+    conv_dirs = {}
     speedup = {}
     n_kernel_groups = 0
     for a in apps:
@@ -623,7 +770,7 @@ def main():
                 kb += b
                 kt += float(r["kernel_ms"])
                 n_kernel_groups += 1
-            c = convert_bytes(a["app"].objects, prec)
+            c = convert_bytes(a["app"].objects, prec, conv_dirs)
             if c:
                 cb += c
                 ct += float(r["convert_ms"])
@@ -646,16 +793,39 @@ def main():
     psrc = (peak_src + " (MEASURED_PEAKS.json hbm_gbs)") if peak_src == "measured" \
         else "fallback (B200_PROFILING.md)"
 
+    # measured DRAM bytes / algorithmic bytes per conversion direction (ncu, 1 GiB launches,
+    # tools/traffic_probe.py -> profiles/ncu_traffic_convert_r2.json), weighted by this
+    # step's bytes per direction
+    conv_ratio, conv_ratio_src = None, None
+    tpc = os.path.join(ROOT, "profiles", "ncu_traffic_convert_r2.json")
+    if os.path.exists(tpc) and conv_dirs:
+        try:
+            dirs = json.load(open(tpc))["directions"]
+            if all(k in dirs for k in conv_dirs):
+                conv_ratio = sum(dirs[k]["ratio"] * v for k, v in conv_dirs.items()) / sum(conv_dirs.values())
+                conv_ratio_src = "profiles/ncu_traffic_convert_r2.json, weighted by %s" % (
+                    {k: round(v / sum(conv_dirs.values()), 4) for k, v in conv_dirs.items()})
+        except Exception:
+            conv_ratio = None
+    if conv_ratio is not None:
+        ratios["convert_ratio"] = conv_ratio
+
     def hbm_roof(bytes_, ms_, n_, kernel, ratio_key):
         if ms_ <= 0 or n_ == 0:
             return None
         ach = bytes_ / (ms_ * 1e-3) / 1e9
         per = bytes_ / n_
         r = ratios.get(ratio_key)
-        return {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "unit": "GB/s",
-                "frac": round(ach / hbm, 4), "traffic": round(r * per) if r else None,
-                "peak_source": psrc, "kernel": kernel,
-                "algorithmic_bytes_per_launch": round(per), "avg_launch_ms": round(ms_ / n_, 5)}
+        out = {"bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "unit": "GB/s",
+               "frac": round(ach / hbm, 4), "traffic": round(r * per) if r else None,
+               "peak_source": psrc, "kernel": kernel,
+               "algorithmic_bytes_per_launch": round(per), "avg_launch_ms": round(ms_ / n_, 5)}
+        if ratio_key == "convert_ratio":
+            out["traffic_source"] = conv_ratio_src or ratios.get("convert_source")
+            out["bytes_by_direction"] = {k: int(v) for k, v in conv_dirs.items()}
+        else:
+            out["traffic_source"] = ratios.get("source")
+        return out
 
     n_conv_groups = sum(1 for a in apps for r in last[a["kind"]]
                         if convert_bytes(a["app"].objects, decode(int(r["config_id"]), a["app"].num_objects)))
@@ -663,7 +833,8 @@ def main():
     roof_a3 = hbm_roof(kb, kt, n_kernel_groups,
                        "a3 statement kernels of one configuration (%s)" % ", ".join(knames), "ratio")
     roof_a2 = hbm_roof(cb, ct, n_conv_groups,
-                       "a2 conversion kernels of one configuration (convert_kernel)", "convert_ratio")
+                       "a2 conversion kernels of one configuration (convert_bulk_kernel: TMA bulk "
+                       "load/store ring)", "convert_ratio")
     roof_mm = contraction_roofline(apps, last) if kb == 0 else None
     roof_st = stencil_roofline(apps, last, hbm)
     # the dominant phase's kernel is THE roofline; the other is reported beside it
@@ -707,7 +878,10 @@ def main():
                    "step": "a0 reference + full 3^M config space per app (a1-a7)",
                    "l2": "inputs larger than L2: largest object %.0f MB at fp32 vs 126 MB L2%s" % (
                        max_obj / 1e6, "" if max_obj > 126e6 else " (NOT larger: launch-bound case)"),
-                   "parallelism": "configs partitioned over %d GPU(s), NCCL result gather" % world},
+                   "parallelism": "configs partitioned over %d GPU(s), NCCL result gather" % world,
+                   "configs_per_rank": per_rank,
+                   "baseline_n_gpus": BASELINE_GPUS.get(args.workload)},
+        "paper_context": PAPER_CONTEXT,
         "e2e": e2e, "gpu_launches": launches,
         "roofline": roof, "cpu_baseline": cpu, "clocks": clk,
         "phase_share": {k: round(v / tot_phase, 4) for k, v in phase.items()} if tot_phase else None,

@@ -65,6 +65,14 @@ PS_API const char *ps_version(void);
 /* Number of CUDA kernels this library has launched in this process (all threads).
  * Used by bench.py to report how many of the library's kernels ran. */
 PS_API uint64_t ps_kernel_launches(void);
+/* 1 when f64 contractions on the current device run on the fp64 tensor-core MMA
+ * (DMMA), 0 when they run on the DFMA kernel.  The DMMA chain is R3's fma chain
+ * bit for bit only if the hardware accumulates one mma.m8n8k4.f64 as a
+ * sequential fma chain (measured on B200, not specified by PTX); the library
+ * checks this on adversarial operands before the first f64 contraction on each
+ * device and falls back to DFMA when it does not hold.  May
+ * synchronise a private stream on first use. */
+PS_API int ps_f64_uses_dmma(void);
 
 /* ------------------------------------------------------------------------- */
 /* (1) Device-side type conversion of one memory object (Fig. 3c). */
@@ -147,9 +155,9 @@ PS_API int ps_app_num_objects(const ps_app *app);            /* -1 if app == NUL
 PS_API ps_status ps_app_object_info(const ps_app *app, int m, ps_object_info *out);
 /* flags: PS_FLAG_NO_TENSOR_CORES forces the SIMT contraction path for fp16   */
 /* operands (bit-exact with R3) instead of tcgen05 (tolerance R6).  It does   */
-/* not concern f64 statements: they always run on the fp64 MMA (mma.sync     */
-/* .f64), whose chained result is R3's fma chain bit for bit (measured,       */
-/* profiles/dmma_probe_r1.txt).                          */
+/* not concern f64 statements: they run on the fp64 MMA (mma.sync.f64) when   */
+/* the per-device self-check shows its chained result is R3's fma chain bit   */
+/* for bit (ps_f64_uses_dmma), else on DFMA chains -- bit-exact either way.   */
 /* PS_FLAG_BF16 extends the configuration alphabet to {f64, f32, f16, bf16}:  */
 /* precision vectors may hold PS_BF16 and ids run over 4^M (radix 4, object 0 */
 /* least significant); without it the space is the paper's 3^M.               */

@@ -27,7 +27,8 @@ ROLE_IN, ROLE_OUT, ROLE_INOUT, ROLE_TEMP = 0, 1, 2, 3
 
 # every symbol include/prescaler.h declares
 SYMBOLS = [
-    "ps_status_string", "ps_last_error", "ps_version", "ps_kernel_launches", "ps_convert",
+    "ps_status_string", "ps_last_error", "ps_version", "ps_kernel_launches", "ps_f64_uses_dmma",
+    "ps_convert",
     "ps_convert_scaled", "ps_quality",
     "ps_app_create", "ps_app_destroy", "ps_app_num_objects", "ps_app_object_info",
     "ps_app_set_flags", "ps_app_workspace_bytes", "ps_app_bind", "ps_app_load_host",
@@ -97,6 +98,7 @@ def lib():
                 "ps_last_error": (ctypes.c_char_p, []),
                 "ps_version": (ctypes.c_char_p, []),
                 "ps_kernel_launches": (ctypes.c_uint64, []),
+                "ps_f64_uses_dmma": (ctypes.c_int, []),
                 "ps_convert": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_int, ctypes.c_size_t, vp]),
                 "ps_convert_scaled": (ctypes.c_int, [vp, ctypes.c_int, vp, ctypes.c_int, ctypes.c_size_t,
                                                      vp, vp]),

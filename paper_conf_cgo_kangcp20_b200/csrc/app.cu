@@ -21,7 +21,10 @@
 #include <atomic>
 #include <chrono>
 #include <map>
+#include <mutex>
+#include <set>
 #include <thread>
+#include <tuple>
 #include <vector>
 
 #include "common.cuh"
@@ -54,6 +57,19 @@ int num_sms() {
     cached[d] = v > 0 ? v : 148;
   }
   return cached[d];
+}
+
+ps_status set_max_smem(const void *kernel, int bytes) {
+  static std::mutex mu;
+  static std::set<std::tuple<int, const void *, int>> done;
+  int d = 0;
+  PS_CUDA(cudaGetDevice(&d));
+  const auto key = std::make_tuple(d, kernel, bytes);
+  std::lock_guard<std::mutex> lk(mu);
+  if (done.count(key)) return PS_OK;
+  PS_CUDA(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+  done.insert(key);
+  return PS_OK;
 }
 
 // ----------------------------------------------------------- app tables
@@ -706,9 +722,9 @@ ps_status enqueue_config(ps_app *a, const int *prec, cudaStream_t st, QPart *res
       out = stage;
       ot = PS_F64;
     }
-    s = backconv_quality_async(out, ot, a->ref[m], a->orig_out[m], nelem(a, m), parts + np, st);
+    s = backconv_quality_async(out, ot, a->ref[m], a->orig_out[m], a->rows[m], a->cols[m], parts + np, st);
     if (s != PS_OK) return s;
-    np += qblocks(nelem(a, m));
+    np += qseg(a->rows[m], a->cols[m]).nb;
   }
   if (ev) PS_CUDA(cudaEventRecord(ev[3], st));
   s = quality_finalize_async(parts, np, res, st);
@@ -1115,6 +1131,14 @@ ps_status ps_run_config_host(ps_app *a, const int *prec, const int *methods,
       return PS_ERR_INVALID;
     }
   }
+  // a->pre[] tells enqueue_config which inputs arrived already converted; it must
+  // be cleared on EVERY exit (a failed transfer must not leave stale markers
+  // that make later ps_run_config / ps_sweep / ps_app_reference skip a2)
+  struct PreReset {
+    ps_app *a;
+    int M;
+    ~PreReset() { for (int m = 0; m < M; m++) a->pre[m] = 0; }
+  } pre_reset{a, M};
   // ---- inputs: host conversion + H2D per object, in object order (wall clock)
   const auto t0 = std::chrono::steady_clock::now();
   for (int m = 0; m < M; m++) {

@@ -26,6 +26,17 @@ ps_status cuda_status(cudaError_t e, const char *what);
     if (_e != cudaSuccess) return ps::cuda_status(_e, #call); \
   } while (0)
 
+#define PS_TRY(expr)                     \
+  do {                                   \
+    ps_status _s = (expr);               \
+    if (_s != PS_OK) return _s;          \
+  } while (0)
+
+// Opt a kernel into `bytes` of dynamic shared memory on the CURRENT device.
+// Thread-safe and per device (the attribute is per device); cheap after the
+// first call for a (device, kernel) pair.
+ps_status set_max_smem(const void *kernel, int bytes);
+
 void count_launch();
 #define PS_CHECK_LAUNCH(what)                                 \
   do {                                                        \

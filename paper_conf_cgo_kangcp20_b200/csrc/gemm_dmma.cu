@@ -262,14 +262,8 @@ template <class SA, class SB, int WGM, int WGN, int BK, int ST, int BN = 128, in
 static ps_status launch_dmma(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
   using C = DCfg<WGM, WGN, BK, ST, BN, MB>;
   constexpr int SM = C::SMEM;
-  static bool attr = false;
-  if (!attr) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST, BN, MB>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
-    PS_CUDA(cudaFuncSetAttribute(gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST, BN, MB>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
-    attr = true;
-  }
+  PS_TRY(set_max_smem((const void *)gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST, BN, MB>, SM));
+  PS_TRY(set_max_smem((const void *)gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST, BN, MB>, SM));
   dim3 grid((unsigned)((p.N + C::BN - 1) / C::BN), (unsigned)((p.M + C::BM - 1) / C::BM));
   if (ak) gemm_dmma_kernel<SA, SB, true, WGM, WGN, BK, ST, BN, MB><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
   else gemm_dmma_kernel<SA, SB, false, WGM, WGN, BK, ST, BN, MB><<<grid, C::THREADS, SM, st>>>(p, alpha, beta, div);
@@ -277,17 +271,16 @@ static ps_status launch_dmma(const Params &p, bool ak, double alpha, double beta
   return PS_OK;
 }
 
-// Variant (measurement switch PS_DMMA_VARIANT; f64 GEMM at 8192^3, profiles/dmma_probe_r1.txt):
-//   0 (default) 128 x 64 CTA tiles of 8 warps (32 x 32 warp tiles), two CTAs per SM,
-//     3 stages of BK 16: 34.2 TFLOP/s
-//   1 128 x 128 tiles of 16 warps, one CTA per SM, 4 stages of BK 16: 29.9
-//   2 128 x 128 tiles of 8 warps (64 x 32 warp tiles), 4 stages of BK 16
-//   3 128 x 128 tiles of 16 warps, 3 stages of BK 32: 31.5
-//   4 128 x 64 tiles, two CTAs per SM, 2 stages of BK 32: 32.3
+// Tile shape history (f64 GEMM at 8192^3, profiles/dmma_probe_r1.txt): 128 x 128 tiles of
+// 16 warps, one CTA per SM, 4 stages of BK 16: 29.9 TFLOP/s; 16 warps, 3 stages of BK 32:
+// 31.5; 128 x 64 tiles, two CTAs per SM, 2 stages of BK 32: 32.3; the shape below: 34.2.
+// The earlier shapes are compiled only with -DPS_LEGACY_KERNELS (PS_DMMA_VARIANT=1..4).
+#ifdef PS_LEGACY_KERNELS
 static int dmma_variant() {
   static const int v = [] { const char *e = getenv("PS_DMMA_VARIANT"); return e ? atoi(e) : 0; }();
   return v;
 }
+#endif
 
 ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st) {
   const Params p = make_params(g);
@@ -296,13 +289,17 @@ ps_status gemm_dmma_f64(const GemmArgs &g, cudaStream_t st) {
     return dispatch_store(g.B.type, [&](auto sb) -> ps_status {
       using SA = decltype(sa);
       using SB = decltype(sb);
+#ifdef PS_LEGACY_KERNELS
       switch (dmma_variant()) {
         case 1: return launch_dmma<SA, SB, 4, 4, 16, 4>(p, ak, g.alpha, g.beta, g.div, st);
         case 2: return launch_dmma<SA, SB, 2, 4, 16, 4>(p, ak, g.alpha, g.beta, g.div, st);
         case 3: return launch_dmma<SA, SB, 4, 4, 32, 3>(p, ak, g.alpha, g.beta, g.div, st);
         case 4: return launch_dmma<SA, SB, 4, 2, 32, 2, 64, 2>(p, ak, g.alpha, g.beta, g.div, st);
-        default: return launch_dmma<SA, SB, 4, 2, 16, 3, 64, 2>(p, ak, g.alpha, g.beta, g.div, st);
+        default: break;
       }
+#endif
+      // 128 x 64 CTA tiles of 8 warps (32 x 32 warp tiles), two CTAs per SM, 3 stages of BK 16
+      return launch_dmma<SA, SB, 4, 2, 16, 3, 64, 2>(p, ak, g.alpha, g.beta, g.div, st);
     });
   });
 }

@@ -192,12 +192,8 @@ __global__ void __launch_bounds__(FTHREADS, 2) gemm_ffma_kernel(Params p, float 
 
 template <class SA, class SB>
 static ps_status launch_ffma(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_ffma_kernel<SA, SB, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM));
-    PS_CUDA(cudaFuncSetAttribute(gemm_ffma_kernel<SA, SB, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM));
-    attr = true;
-  }
+  PS_TRY(set_max_smem((const void *)gemm_ffma_kernel<SA, SB, true>, FSMEM));
+  PS_TRY(set_max_smem((const void *)gemm_ffma_kernel<SA, SB, false>, FSMEM));
   dim3 grid((unsigned)((p.N + FBN - 1) / FBN), (unsigned)((p.M + FBM - 1) / FBM));
   // scalars are RNE-rounded from their fp64 literal to f32 (R2); the host cast is RNE
   if (ak) gemm_ffma_kernel<SA, SB, true><<<grid, FTHREADS, FSMEM, st>>>(p, (float)alpha, (float)beta, (float)div);

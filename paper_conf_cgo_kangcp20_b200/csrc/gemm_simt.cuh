@@ -257,12 +257,8 @@ template <class T, class SA, class SB>
 ps_status launch(const Params &p, bool ak, double alpha, double beta, double div, cudaStream_t st) {
   using C = Cfg<T>;
   constexpr int SM = smem_bytes<T>();
-  static bool attr = false;
-  if (!attr) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_kernel<T, SA, SB, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
-    PS_CUDA(cudaFuncSetAttribute(gemm_kernel<T, SA, SB, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, SM));
-    attr = true;
-  }
+  PS_TRY(set_max_smem((const void *)gemm_kernel<T, SA, SB, true>, SM));
+  PS_TRY(set_max_smem((const void *)gemm_kernel<T, SA, SB, false>, SM));
   dim3 grid((unsigned)((p.N + C::BN - 1) / C::BN), (unsigned)((p.M + C::BM - 1) / C::BM));
   // scalars are RNE-rounded from their fp64 literal to T (R2); the host cast is RNE
   if (ak) gemm_kernel<T, SA, SB, true><<<grid, C::THREADS, SM, st>>>(p, (T)alpha, (T)beta, (T)div);

@@ -43,7 +43,7 @@ constexpr int EPI_COLS = 32;
 constexpr int EPI_STRIDE = 36;                                // floats per staged row (conflict-free float4)
 // 8 epilogue warps: two per TMEM lane quarter (warp w may read lanes 32 (w % 4)..),
 // each draining half of the accumulator's columns -- twice the memory-level
-// parallelism of one warp per quarter, which paced the fp8 tiles (ncu / PS_TC_NOEPI)
+// parallelism of one warp per quarter, which paced the fp8 tiles (ncu, round 1)
 constexpr int EPI_WARPS = 8;
 constexpr int EPI_SMEM = EPI_WARPS * 32 * EPI_STRIDE * 4;     // 36 KiB
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + EPI_SMEM;
@@ -73,7 +73,6 @@ struct Params {
   uint32_t a_fmt, b_fmt;   // kind::f16: 0 = f16, 1 = bf16 (reading #28); kind::f8f6f4: 0 = E4M3, 1 = E5M2
   const ps_fp8_scale *sa, *sb;   // fp8 operands: per-tensor scales (reading #29)
   int vec4;                // C / Cin rows 4-element aligned: vector epilogue stores / loads
-  int noepi;               // experiment (PS_TC_NOEPI): skip the epilogue's stores (results invalid)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -199,7 +198,6 @@ __device__ __forceinline__ float epi_op(const Params &p, float r, float cin) {
 // the matching Cin load for alpha/beta).  fp8 operands: accumulator x 2^kab first.
 __device__ __forceinline__ void epi_chunk(const Params &p, float *stg, int lane, int64_t row0,
                                           int64_t col0, const uint32_t (&v)[32], int kab) {
-  if (p.noepi) return;
   float4 *srow = reinterpret_cast<float4 *>(stg + lane * EPI_STRIDE);
 #pragma unroll
   for (int q = 0; q < 8; q++)
@@ -691,11 +689,7 @@ template <int ES>
 static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   using namespace tc;
   using G = Geo<ES>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    PS_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<ES>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES));
-    attr_set = true;
-  }
+  PS_TRY(set_max_smem((const void *)gemm_tc_kernel<ES>, SMEM_BYTES));
   CUtensorMap ma, mb;
   const bool a_mn = !(g.A.s_col == 1);
   const bool b_k = !(g.B.s_col == 1);
@@ -714,7 +708,7 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   const uint32_t bfm = (g.B.type == PS_BF16 || g.B.type == PS_E5M2) ? 1u : 0u;
   Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, b_k ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
            (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, af, bfm,
-           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr, 0, getenv("PS_TC_NOEPI") ? 1 : 0};
+           ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr, 0};
   {   // vector epilogue: rows of C (and Cin) start 16-byte (f32) / 8-byte (16-bit) aligned
     const int64_t cb = (int64_t)dtype_size(g.c_type);
     bool v4 = g.ldc % 4 == 0 && (uintptr_t)g.C % (4 * cb) == 0;
@@ -723,12 +717,7 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   }
   if (two) {   // 2-CTA persistent path
     using namespace tc2;
-    static bool attr2 = false;
-    if (!attr2) {
-      PS_CUDA(cudaFuncSetAttribute(gemm_tc2_kernel<ES>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   tc2::SMEM_BYTES));
-      attr2 = true;
-    }
+    PS_TRY(set_max_smem((const void *)gemm_tc2_kernel<ES>, tc2::SMEM_BYTES));
     Sched sch;
     sch.tiles_m = (g.M + tc2::BM - 1) / tc2::BM;
     sch.tiles_n = (g.N + tc2::BN - 1) / tc2::BN;
@@ -750,43 +739,7 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   return PS_OK;
 }
 
-// out[j * K + k] = in[k * ld + j]: an N-major K x N operand copied K-contiguous
-template <class E>
-__global__ void __launch_bounds__(256) transpose_kernel(const E *__restrict__ in, E *__restrict__ out,
-                                                        int64_t K, int64_t N, int64_t ld) {
-  __shared__ E t[32][33];
-  const int64_t k0 = (int64_t)blockIdx.y * 32, j0 = (int64_t)blockIdx.x * 32;
-  for (int r = threadIdx.y; r < 32; r += 8) {
-    const int64_t k = k0 + r, j = j0 + threadIdx.x;
-    if (k < K && j < N) t[r][threadIdx.x] = in[k * ld + j];
-  }
-  __syncthreads();
-  for (int r = threadIdx.y; r < 32; r += 8) {
-    const int64_t j = j0 + r, k = k0 + threadIdx.x;
-    if (k < K && j < N) out[j * K + k] = t[threadIdx.x][r];
-  }
-}
-
-ps_status gemm_tc_async(const GemmArgs &g0, cudaStream_t st) {
-  GemmArgs g = g0;
-  static const bool bt = getenv("PS_TC_BT") != nullptr;   // experiment: K-major B via a transposed copy
-  if (bt && g.B.s_col == 1 && g.K % 16 == 0) {
-    static void *buf = nullptr;
-    static size_t cap = 0;
-    const size_t es = dtype_size(g.B.type), need = (size_t)g.K * (size_t)g.N * es;
-    if (need > cap) {
-      if (buf) cudaFree(buf);
-      PS_CUDA(cudaMalloc(&buf, need));
-      cap = need;
-    }
-    const dim3 grid((unsigned)((g.N + 31) / 32), (unsigned)((g.K + 31) / 32)), blk(32, 8);
-    if (es == 1) transpose_kernel<uint8_t><<<grid, blk, 0, st>>>((const uint8_t *)g.B.p, (uint8_t *)buf, g.K, g.N, g.B.s_row);
-    else transpose_kernel<uint16_t><<<grid, blk, 0, st>>>((const uint16_t *)g.B.p, (uint16_t *)buf, g.K, g.N, g.B.s_row);
-    PS_CHECK_LAUNCH("transpose_kernel");
-    g.B.p = buf;
-    g.B.s_row = 1;
-    g.B.s_col = g.K;
-  }
+ps_status gemm_tc_async(const GemmArgs &g, cudaStream_t st) {
   return is_fp8(g.A.type) ? gemm_tc_launch<1>(g, st) : gemm_tc_launch<2>(g, st);
 }
 

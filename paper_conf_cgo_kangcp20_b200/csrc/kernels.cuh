@@ -24,10 +24,18 @@ struct QPart {
   double mx;
   unsigned long long nf;
 };
-int qblocks(size_t n);
+// segments of a rows x cols output: `per` elements each (whole rows when rows > 1)
+struct QSeg {
+  int64_t per;        // elements per segment
+  int64_t rows_per;   // rows per segment (1 for a vector)
+  int nb;             // segments (<= QBLOCKS_MAX)
+};
+QSeg qseg(int64_t rows, int64_t cols);
+// segments [seg0, seg1) (seg1 < 0: all) of the output; partial of segment k -> parts[k];
 // delivered == nullptr: score the exact widened value, no write (ps_quality)
 ps_status backconv_quality_async(const void *out, int out_type, const double *ref, float *delivered,
-                                 size_t n, QPart *parts, cudaStream_t st);
+                                 int64_t rows, int64_t cols, QPart *parts, cudaStream_t st,
+                                 int seg0 = 0, int seg1 = -1);
 ps_status quality_finalize_async(const QPart *parts, int nparts, QPart *res, cudaStream_t st);
 
 // ------------------------------------------------------ contractions (a3)

@@ -7,9 +7,12 @@
 //   e = 0 if o == r; 1 if o or r non-finite or r == 0; else min(1, |o-r|/|r|)
 // One read of out_c and ref, one write of the delivered f32 output; sum(e) in
 // fp64, max of the uncapped relative error, count of non-finite o.
-// Deterministic: the element->thread map depends on n only (fixed grid size
-// QBLOCKS(n), fixed block size, fixed shuffle/smem trees), never on the SM
-// count, so results are bit-identical across GPUs and rank counts.
+// Deterministic: the output (rows x cols) is cut into QSeg segments that depend
+// on its shape only -- whole rows for a matrix (so a row-sharded evaluation,
+// ps_shard_step, computes exactly the segments of its rows), ~equal pieces of a
+// vector -- one block per segment with a fixed thread map and fixed shuffle/smem
+// trees, never on the SM count; the finalize adds the segment partials in
+// segment order.  So results are bit-identical across GPUs and rank counts.
 #include <math.h>
 
 #include "common.cuh"
@@ -85,16 +88,19 @@ __device__ __forceinline__ void block_reduce3(double &sum, double &mx, unsigned 
 }
 
 // DELIVER: round to the original precision f32 and write it (pipeline, a4);
-// otherwise score the exact widened value (standalone ps_quality).
+// otherwise score the exact widened value (standalone ps_quality).  Block b
+// handles segment seg0 + b = elements [seg * per, min(n, (seg + 1) * per)).
 template <class S, bool DELIVER>
 __global__ void __launch_bounds__(QTHREADS) backconv_quality_kernel(
     const raw_t<S> *__restrict__ out, const double *__restrict__ ref, float *__restrict__ delivered,
-    size_t n, QPart *__restrict__ parts) {
+    size_t n, size_t per, int seg0, QPart *__restrict__ parts) {
   __shared__ double s_sum[QTHREADS / 32], s_mx[QTHREADS / 32];
   __shared__ unsigned long long s_nf[QTHREADS / 32];
   double sum = 0.0, mx = 0.0;
   unsigned long long nf = 0;
-  const size_t stride = (size_t)gridDim.x * QTHREADS;
+  const int seg = seg0 + (int)blockIdx.x;
+  const size_t base = (size_t)seg * per;
+  const size_t end = base + per < n ? base + per : n;
   auto one = [&](size_t i, raw_t<S> v, double r) {
     double o;
     if (DELIVER) {
@@ -108,11 +114,11 @@ __global__ void __launch_bounds__(QTHREADS) backconv_quality_kernel(
   };
   // 4 consecutive elements per thread per step: 16-byte loads of ref (2 x double2)
   // and of out (f32) / 8-byte (f16) / 2 x 16-byte (f64) when everything is aligned
-  const bool vec = ((uintptr_t)out % 16 == 0) && ((uintptr_t)ref % 16 == 0) &&
+  const bool vec = base % 4 == 0 && ((uintptr_t)out % 16 == 0) && ((uintptr_t)ref % 16 == 0) &&
                    (!DELIVER || (uintptr_t)delivered % 16 == 0);
-  size_t i = ((size_t)blockIdx.x * QTHREADS + threadIdx.x) * 4;
+  size_t i = base + (size_t)threadIdx.x * 4;
   if (vec) {
-    for (; i + 4 <= n; i += stride * 4) {
+    for (; i + 4 <= end; i += (size_t)QTHREADS * 4) {
       const double2 r0 = __ldg(reinterpret_cast<const double2 *>(ref + i));
       const double2 r1 = __ldg(reinterpret_cast<const double2 *>(ref + i) + 1);
       raw_t<S> v[4];
@@ -136,13 +142,12 @@ __global__ void __launch_bounds__(QTHREADS) backconv_quality_kernel(
         qual_elem(Deliver<S>::exact(v[3]), r1.y, sum, mx, nf);
       }
     }
-    for (; i < n; i++) one(i, out[i], __ldg(ref + i));   // ragged tail (this thread's last group)
+    for (; i < end; i++) one(i, out[i], __ldg(ref + i));   // ragged tail (this thread's last group)
   } else {
-    for (size_t e = (size_t)blockIdx.x * QTHREADS + threadIdx.x; e < n; e += stride)
-      one(e, out[e], __ldg(ref + e));
+    for (size_t e = base + threadIdx.x; e < end; e += QTHREADS) one(e, out[e], __ldg(ref + e));
   }
   block_reduce3(sum, mx, nf, s_sum, s_mx, s_nf);
-  if (threadIdx.x == 0) parts[blockIdx.x] = QPart{sum, mx, nf};
+  if (threadIdx.x == 0) parts[seg] = QPart{sum, mx, nf};
 }
 
 // Sums nparts partials in a fixed order into *res (one block).
@@ -162,23 +167,44 @@ __global__ void __launch_bounds__(QTHREADS) quality_finalize_kernel(const QPart 
   if (threadIdx.x == 0) *res = QPart{sum, mx, nf};
 }
 
-int qblocks(size_t n) {
-  size_t b = (n + (size_t)QTHREADS * 4 - 1) / ((size_t)QTHREADS * 4);
-  if (b > (size_t)QBLOCKS_MAX) b = QBLOCKS_MAX;
-  return b ? (int)b : 1;
+QSeg qseg(int64_t rows, int64_t cols) {
+  QSeg q;
+  const int64_t n = rows * cols;
+  if (n <= 0) return QSeg{1, 1, 1};
+  if (rows > 1) {   // whole rows: >= ~1024 elements per segment, <= QBLOCKS_MAX segments
+    int64_t rps = (rows + QBLOCKS_MAX - 1) / QBLOCKS_MAX;
+    const int64_t want = (1024 + cols - 1) / cols;
+    if (rps < want) rps = want;
+    if (rps > rows) rps = rows;
+    q.rows_per = rps;
+    q.per = rps * cols;
+  } else {          // a vector: ~equal pieces of 4 * QTHREADS-element multiples
+    int64_t nb = (n + (int64_t)QTHREADS * 4 - 1) / ((int64_t)QTHREADS * 4);
+    if (nb > QBLOCKS_MAX) nb = QBLOCKS_MAX;
+    int64_t per = (n + nb - 1) / nb;
+    per = (per + 3) / 4 * 4;
+    q.rows_per = 1;
+    q.per = per;
+  }
+  q.nb = (int)((n + q.per - 1) / q.per);
+  return q;
 }
 
 ps_status backconv_quality_async(const void *out, int out_type, const double *ref, float *delivered,
-                                 size_t n, QPart *parts, cudaStream_t st) {
-  const int nb = qblocks(n);
+                                 int64_t rows, int64_t cols, QPart *parts, cudaStream_t st, int seg0,
+                                 int seg1) {
+  const QSeg q = qseg(rows, cols);
+  if (seg1 < 0 || seg1 > q.nb) seg1 = q.nb;
+  if (seg0 >= seg1) return PS_OK;
+  const size_t n = (size_t)(rows * cols);
   auto go = [&](auto s) -> ps_status {
     using S = decltype(s);
     if (delivered)
-      backconv_quality_kernel<S, true><<<nb, QTHREADS, 0, st>>>((const raw_t<S> *)out, ref,
-                                                               delivered, n, parts);
+      backconv_quality_kernel<S, true><<<seg1 - seg0, QTHREADS, 0, st>>>(
+          (const raw_t<S> *)out, ref, delivered, n, (size_t)q.per, seg0, parts);
     else
-      backconv_quality_kernel<S, false><<<nb, QTHREADS, 0, st>>>((const raw_t<S> *)out, ref,
-                                                                nullptr, n, parts);
+      backconv_quality_kernel<S, false><<<seg1 - seg0, QTHREADS, 0, st>>>(
+          (const raw_t<S> *)out, ref, nullptr, n, (size_t)q.per, seg0, parts);
     PS_CHECK_LAUNCH("backconv_quality_kernel");
     return PS_OK;
   };
@@ -240,9 +266,9 @@ extern "C" ps_status ps_quality(const void *out, int out_type, const double *ref
     ps_status s = scratch_get(&dev, &host);
     if (s != PS_OK) return s;
     cudaStream_t st = (cudaStream_t)stream;
-    s = backconv_quality_async(out, out_type, ref, nullptr, n, dev + 1, st);
+    s = backconv_quality_async(out, out_type, ref, nullptr, 1, (int64_t)n, dev + 1, st);
     if (s != PS_OK) return s;
-    s = quality_finalize_async(dev + 1, qblocks(n), dev, st);
+    s = quality_finalize_async(dev + 1, qseg(1, (int64_t)n).nb, dev, st);
     if (s != PS_OK) return s;
     PS_CUDA(cudaMemcpyAsync(host, dev, sizeof(QPart), cudaMemcpyDeviceToHost, st));
     PS_CUDA(cudaStreamSynchronize(st));

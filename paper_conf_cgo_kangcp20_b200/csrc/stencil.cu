@@ -304,12 +304,7 @@ ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64
       constexpr bool SAME = std::is_same<raw_t<SA>, T>::value;
       const size_t smem = (sizeof(T) * C3_RING + (SAME ? 0 : 2 * sizeof(raw_t<SA>))) * C3_SH * C3Geo<SA>::SW;
       const int vec_ok = ((uintptr_t)A % 16 == 0) && ((nk * (int64_t)sizeof(raw_t<SA>)) % 16 == 0);
-      static bool attr[3][3];                          // per instantiation, set once
-      if (!attr[Store<SA>::code][Store<SB>::code]) {
-        PS_CUDA(cudaFuncSetAttribute(conv3d_kernel<SA, SB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)smem));
-        attr[Store<SA>::code][Store<SB>::code] = true;
-      }
+      PS_TRY(set_max_smem((const void *)conv3d_kernel<SA, SB>, (int)smem));
       conv3d_kernel<SA, SB><<<grid, C3_NT, smem, st>>>((const raw_t<SA> *)A, (raw_t<SB> *)B, ni, nj, nk, cf,
                                                          vec_ok);
       PS_CHECK_LAUNCH("conv3d_kernel");

@@ -17,6 +17,8 @@
 // algorithmic bytes = R*C*sizeof(A) per pass + O(R + C).
 #include <math.h>
 
+#include <atomic>
+
 #include <type_traits>
 
 #include "common.cuh"
@@ -246,10 +248,12 @@ size_t tile_partial_bytes(int64_t rows, int64_t cols) {
 
 template <class SA, class TC, class TR, int CM, bool RD>
 static ps_status launch_tile(const TileArgs &a, cudaStream_t st) {
-  static int occ = 0;
+  static std::atomic<int> occ_cache{0};   // same for every B200 of the box
+  int occ = occ_cache.load(std::memory_order_relaxed);
   if (!occ) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tile_kernel<SA, TC, TR, CM, RD>, TTHREADS, 0);
     if (occ < 1) occ = 1;
+    occ_cache.store(occ, std::memory_order_relaxed);
   }
   const int64_t cap = (int64_t)num_sms() * occ;
   int64_t gy = cap / a.ntiles;

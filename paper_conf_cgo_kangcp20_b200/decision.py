@@ -190,14 +190,21 @@ def decide(app, host_inputs, db: dict, toq: float = 0.9, threads: int = 0, verif
                 if wbest is None or expected < wbest[2]:
                     wbest = (prec, meth, expected, inter)
             if wbest is not None and wbest[2] < best_r["total_ms"]:        # line 23
-                prec, meth, _, inter = wbest
-                ok = True
+                prec, meth, expected, inter = wbest
                 if verify or inter == failed:                                # lines 24-28
-                    ok = run_app(prec, meth)["pass"]
-                if ok:
+                    # measured: keep it only if it passes AND beats the measured best
+                    r = run_app(prec, meth)
+                    if r["pass"] and r["total_ms"] < best_r["total_ms"]:
+                        best, best_m, best_r = prec, meth, r
+                else:
+                    # Alg. 1 accepts on the expected time without a RunApp call when
+                    # the transient intermediate is not the type that failed
                     best, best_m = prec, meth
-                    best_r = run_app(prec, meth)
+                    best_r = {"total_ms": expected, "pass": True, "expected_only": True,
+                              "kernel_side_ms": kernel_ms.get(prec[k], float("inf"))}
         cur, cur_m, cur_r = best, best_m, best_r
+    if cur_r.get("expected_only"):                 # the final report needs a measured run
+        cur_r = run_app(cur, cur_m)
 
     return {"prec": list(cur), "methods": list(cur_m), "method_names": [NAMES[m] for m in cur_m],
             "result": cur_r, "pfp": pfp, "trials": len(log), "log": log,

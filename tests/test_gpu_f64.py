@@ -66,11 +66,17 @@ def test_f64_statements_bit_exact_adversarial(torch, kind, dims, sc):
             check_config(torch, app, kind, dims, ins, oref, prec, sc)
 
 
-@pytest.mark.parametrize("switch", ["PS_F64_DFMA", "PS_F32_SIMT_OLD"])
-def test_previous_kernels_bit_exact(switch):
-    """The kernels kept behind measurement switches (the DFMA f64 kernel, PS_F64_DFMA=1;
-    the previous FFMA kernel, PS_F32_SIMT_OLD=1) stay R3-exact: the contraction apps'
-    exhaustive SIMT parity cases in a child process."""
+def test_dmma_self_check_selects_dmma_on_b200():
+    """ps_f64_uses_dmma: the per-device self-check (adversarial 128x128x64 product,
+    DMMA vs DFMA bit for bit) passes on B200, so f64 statements run on DMMA."""
+    from paper_conf_cgo_kangcp20_b200 import binding as B
+    assert B.lib().ps_f64_uses_dmma() == 1
+
+
+@pytest.mark.parametrize("switch", ["PS_F64_DFMA"])
+def test_fallback_kernel_bit_exact(switch):
+    """The DFMA f64 kernel (the self-check fallback, forced by PS_F64_DFMA=1) stays
+    R3-exact: the contraction apps' exhaustive SIMT parity cases in a child process."""
     env = dict(os.environ, **{switch: "1"})
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-p", "no:cacheprovider", "-m", "gpu",
                         os.path.join(ROOT, "tests", "test_gpu_apps.py"),
