@@ -240,6 +240,51 @@ PS_API ps_status ps_config_decode(const ps_app *app, uint64_t id, int *prec);
 PS_API ps_status ps_run_config(ps_app *app, const int *prec, double toq, void *stream, ps_result *out);
 
 /* ------------------------------------------------------------------------- */
+/* (4b) ONE configuration evaluated by W ranks, each owning a contiguous range  */
+/*   of the app's sharded rows ("very large memory objects        */
+/*   sharded by contiguous range"; north star item 5).  The sharded dimension:  */
+/*   the rows of A (and B) for ATAX / BICG / GESUMMV / MVT; the rows of the      */
+/*   scored output for GEMM, 2MM, 3MM (F rows get their own split), SYR2K,     */
+/*   2DCONV, 3DCONV; the upper-triangular output rows for SYRK, CORR, COVAR     */
+/*   (CORR / COVAR split the data rows for the column statistics).  FDTD-2D     */
+/*   (TMAX dependent sweeps) and fp8 objects (per-tensor scales need the whole */
+/*   object) are not row-shardable: PS_ERR_UNSUPPORTED.                         */
+/*   Row bounds are aligned so every reduction keeps its single-GPU association */
+/*   (R5 256-row column-sum chunks, whole quality segments, whole 256-row      */
+/*   tcgen05 tiles): the record and the delivered outputs are bit-identical to */
+/*   ps_run_config for every W.  Protocol, on every rank r of W:               */
+/*     for (stage = 0; ; stage++) {                                            */
+/*       ps_shard_step(app, prec, toq, r, W, stage, stream, &x);               */
+/*       if (x.done) break;             // x.result is the configuration's record */
+/*       for k < x.nregions: copy this rank's bytes [off, off + len) of        */
+/*         x.region[k].ptr to the same offsets on every other rank (each rank's */
+/*         (off, len) differ; e.g. an NCCL all-gather of padded pieces)        */
+/*     }                                                                        */
+/*   region.ptr is a device pointer into this rank's workspace (same layout on */
+/*   every rank).  Delivered outputs: the rows the rank owns of a row-sharded  */
+/*   output, every element of vector outputs.  ps_shard_step synchronises      */
+/*   `stream` at the end of each stage; result times are summed over stages    */
+/*   (device work only, exchanges excluded).  One configuration at a time per */
+/*   app (stages keep state in the workspace).                                  */
+typedef struct {
+  void *ptr;      /* device buffer in the workspace                        */
+  uint64_t off;   /* this rank's byte range [off, off + len) of ptr        */
+  uint64_t len;
+} ps_shard_region;
+typedef struct {
+  int32_t done;       /* 1: evaluation complete, `result` valid          */
+  int32_t nregions;   /* regions to exchange before the next stage (<= 4) */
+  ps_shard_region region[4];
+  ps_result result;
+} ps_shard_step_t;
+/* rows of the sharded dimension, 0 = the app has no row-sharded evaluation */
+PS_API int64_t ps_app_eval_shard_rows(const ps_app *app);
+/* rank's row range [*row0, *row1) of that dimension among `world` ranks (may be empty) */
+PS_API ps_status ps_shard_bounds(const ps_app *app, int rank, int world, int64_t *row0, int64_t *row1);
+PS_API ps_status ps_shard_step(ps_app *app, const int *prec, double toq, int rank, int world, int stage,
+                               void *stream, ps_shard_step_t *x);
+
+/* ------------------------------------------------------------------------- */
 /* (5) Evaluate a list of configuration ids (a7).  results[i] for config_ids[i] */
 /* (host array).  *best_index = index of the fastest passing config (ties ->   */
 /* lowest id), -1 if none passes.  One stream synchronisation at the end.      */

@@ -992,13 +992,50 @@ static void stats_column(int corr, obj_t *data, obj_t *mean, obj_t *sd, size_t N
   }
 }
 
+/* Sampling speed only (no arithmetic change): the exact values of o[0..n), as ld
+ * returns them, cached in o->val so repeated loads skip the software widening.
+ * The object must not be stored to while cached (ld prefers val). */
+static double *cache_values(obj_t *o) {
+  size_t i;
+  double *buf = (double *)malloc(sizeof(double) * (o->n ? o->n : 1));
+  o->val = NULL;
+  for (i = 0; i < o->n; i++) buf[i] = ld(o, i);
+  o->val = buf;
+  return buf;
+}
+
+/* sorted distinct values of v[0..n): out[0] = count, out[1..] = values (malloc) */
+static int cmp_i64(const void *x, const void *y) {
+  int64_t a = *(const int64_t *)x, b = *(const int64_t *)y;
+  return a < b ? -1 : (a > b ? 1 : 0);
+}
+static int64_t *uniq(const int64_t *v, size_t n, void *unused) {
+  int64_t *o = (int64_t *)malloc(sizeof(int64_t) * (n + 1));
+  size_t k, c = 0;
+  (void)unused;
+  if (n) memcpy(o + 1, v, sizeof(int64_t) * n);
+  qsort(o + 1, n, sizeof(int64_t), cmp_i64);
+  for (k = 0; k < n; k++)
+    if (c == 0 || o[1 + k] != o[c]) o[1 + c++] = o[1 + k];
+  o[0] = (int64_t)c;
+  return o;
+}
+static size_t uniq_index(const int64_t *u, int64_t x) {
+  size_t lo = 0, hi = (size_t)u[0];
+  while (lo + 1 < hi) {
+    size_t mid = (lo + hi) / 2;
+    if (u[1 + mid] <= x) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
 int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double *sc,
                   const int *prec, const float *const *inputs, int m, const int64_t *rows,
                   const int64_t *cols, size_t n, double *vals) {
   const app_def_t *a = find_app(kind);
   int64_t d[8], R[8], C[8];
   obj_t in[8];
-  size_t k, q;
+  size_t k;
   int t;
   if (!a || full_dims(a, dims, ndims, d) || !prec || m < 0 || m >= a->nobj || !a->outputs[m] ||
       (n && (!rows || !cols || !vals)))
@@ -1016,6 +1053,9 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
   }
   for (k = 0; k < n; k++)
     if (rows[k] < 0 || rows[k] >= R[m] || cols[k] < 0 || cols[k] >= C[m]) return 1;
+  if (strcmp(kind, "fdtd2d"))
+    for (t = 0; t < a->nobj; t++)
+      if (in[t].src) cache_values(&in[t]);
 
   if (!strcmp(kind, "gemm")) {
     size_t NJ = d[1], NK = d[2];
@@ -1035,32 +1075,43 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
     for (k = 0; k < n; k++) {
       size_t i = rows[k], l = cols[k];
       if ((int64_t)i != cached) {           /* row i of C <- A . B */
+        free(crow.val);
+        crow.val = NULL;
         for (j = 0; j < NJ; j++) st(&crow, j, dot_chain(T1, &in[0], i * NK, 1, &in[1], j, NJ, NK), T1);
+        cache_values(&crow);
         cached = (int64_t)i;
       }
       vals[k] = round_to(prec[4], dot_chain(T2, &crow, 0, 1, &in[3], l, NL, NJ), T2);
     }
     free(crow.p);
+    free(crow.val);
   } else if (!strcmp(kind, "3mm")) {
-    size_t NJ = d[1], NK = d[2], NL = d[3], NM = d[4], j;
+    /* every distinct row i of E <- A . B and column l of F <- C . D is computed
+     * once (no arithmetic difference: each is the same R3 chain) */
+    size_t NJ = d[1], NK = d[2], NL = d[3], NM = d[4], j, u;
     int T1 = W3(prec[0], prec[1], prec[4]), T2 = W3(prec[2], prec[3], prec[5]);
     int T3 = W3(prec[4], prec[5], prec[6]);
-    obj_t erow = new_obj(prec[4], NJ), fcol = new_obj(prec[5], NJ);
-    int64_t ci = -1, cl = -1;
+    int64_t *ur = uniq(rows, n, NULL), *uc = uniq(cols, n, NULL);
+    size_t nr = (size_t)ur[0], nc = (size_t)uc[0];
+    obj_t erows = new_obj(prec[4], nr * NJ), fcols = new_obj(prec[5], nc * NJ);
+    for (u = 0; u < nr; u++)
+      for (j = 0; j < NJ; j++)
+        st(&erows, u * NJ + j, dot_chain(T1, &in[0], (size_t)ur[1 + u] * NK, 1, &in[1], j, NJ, NK), T1);
+    for (u = 0; u < nc; u++)
+      for (j = 0; j < NJ; j++)
+        st(&fcols, u * NJ + j, dot_chain(T2, &in[2], j * NM, 1, &in[3], (size_t)uc[1 + u], NL, NM), T2);
+    cache_values(&erows);
+    cache_values(&fcols);
     for (k = 0; k < n; k++) {
-      size_t i = rows[k], l = cols[k];
-      if ((int64_t)i != ci) {               /* row i of E <- A . B */
-        for (j = 0; j < NJ; j++) st(&erow, j, dot_chain(T1, &in[0], i * NK, 1, &in[1], j, NJ, NK), T1);
-        ci = (int64_t)i;
-      }
-      if ((int64_t)l != cl) {               /* column l of F <- C . D */
-        for (j = 0; j < NJ; j++) st(&fcol, j, dot_chain(T2, &in[2], j * NM, 1, &in[3], l, NL, NM), T2);
-        cl = (int64_t)l;
-      }
-      vals[k] = round_to(prec[6], dot_chain(T3, &erow, 0, 1, &fcol, 0, 1, NJ), T3);
+      size_t ri = uniq_index(ur, rows[k]), li = uniq_index(uc, cols[k]);
+      vals[k] = round_to(prec[6], dot_chain(T3, &erows, ri * NJ, 1, &fcols, li * NJ, 1, NJ), T3);
     }
-    free(erow.p);
-    free(fcol.p);
+    free(erows.p);
+    free(fcols.p);
+    free(erows.val);
+    free(fcols.val);
+    free(ur);
+    free(uc);
   } else if (!strcmp(kind, "atax")) {
     size_t NX = d[0], NY = d[1], i;
     int T1 = W3(prec[0], prec[1], prec[3]), T2 = W3(prec[0], prec[3], prec[2]);
@@ -1142,26 +1193,47 @@ int oracle_sample(const char *kind, const int64_t *dims, int ndims, const double
     for (k = 0; k < n; k++) vals[k] = ld(&o[m], (size_t)(rows[k] * C[m] + cols[k]));
     free_objects(o, ap->nobj);
   } else {                                  /* corr / covar: symmat entries */
+    /* column j of the normalised (CORR) / centred (COVAR) data is computed once
+     * per distinct j (no arithmetic difference: stats_column is per column) */
     int corr = !strcmp(kind, "corr");
-    size_t N = d[0], M = d[1];
+    size_t N = d[0], M = d[1], u;
     int so = corr ? 3 : 2;
     obj_t mean = new_obj(prec[1], M), sd = new_obj(corr ? prec[2] : OR_F64, M);
-    obj_t z1 = new_obj(prec[0], N), z2 = new_obj(prec[0], N);
+    obj_t z = new_obj(prec[0], N);
     int T = W2(prec[0], prec[so]);
     double eps = scalar_or(sc, 0, 0.005);
+    int64_t *lo = (int64_t *)malloc(sizeof(int64_t) * (n ? n : 1));
+    int64_t *hi = (int64_t *)malloc(sizeof(int64_t) * (n ? n : 1));
+    int64_t *both = (int64_t *)malloc(sizeof(int64_t) * (2 * n + 1));
+    int64_t *uz;
+    obj_t zc;
     for (k = 0; k < n; k++) {
-      size_t j1 = rows[k], j2 = cols[k];
-      if (j1 > j2) { size_t s = j1; j1 = j2; j2 = s; }   /* mirrored lower triangle */
+      lo[k] = rows[k] < cols[k] ? rows[k] : cols[k];   /* mirrored lower triangle */
+      hi[k] = rows[k] < cols[k] ? cols[k] : rows[k];
+      both[k] = lo[k];
+      both[n + k] = hi[k];
+    }
+    uz = uniq(both, 2 * n, NULL);
+    zc = new_obj(prec[0], (size_t)uz[0] * N);
+    for (u = 0; u < (size_t)uz[0]; u++) {
+      size_t i;
+      stats_column(corr, &in[0], &mean, &sd, N, M, (size_t)uz[1 + u], eps, &z);
+      for (i = 0; i < N; i++) st(&zc, u * N + i, ld(&z, i), prec[0] == OR_F64 ? OR_F64 : OR_F32);
+    }
+    cache_values(&zc);
+    for (k = 0; k < n; k++) {
+      size_t j1 = (size_t)lo[k], j2 = (size_t)hi[k];
       if (corr && j1 == j2) { vals[k] = round_to(prec[so], 1.0, T); continue; }
-      stats_column(corr, &in[0], &mean, &sd, N, M, j1, eps, &z1);
-      stats_column(corr, &in[0], &mean, &sd, N, M, j2, eps, &z2);
       {
-        double acc = dot_chain(T, &z1, 0, 1, &z2, 0, 1, N);
+        size_t a1 = uniq_index(uz, (int64_t)j1), a2 = uniq_index(uz, (int64_t)j2);
+        double acc = dot_chain(T, &zc, a1 * N, 1, &zc, a2 * N, 1, N);
         if (!corr) acc = t_div(T, acc, t_lit(T, (double)N - 1.0));
         vals[k] = round_to(prec[so], acc, T);
       }
     }
-    for (q = 0; q < 1; q++) { free(mean.p); free(sd.p); free(z1.p); free(z2.p); }
+    free(mean.p); free(sd.p); free(z.p); free(zc.p); free(zc.val);
+    free(lo); free(hi); free(both); free(uz);
   }
+  for (t = 0; t < a->nobj; t++) free(in[t].val);
   return 0;
 }

@@ -35,7 +35,7 @@ SYMBOLS = [
     "ps_app_reference", "ps_app_set_reference", "ps_config_encode", "ps_config_decode",
     "ps_run_config", "ps_sweep", "ps_search", "ps_host_convert", "ps_run_config_host",
     "ps_transfer", "ps_app_shard_rows", "ps_app_shard_triangular", "ps_app_reference_rows",
-    "ps_app_reference_merge",
+    "ps_app_reference_merge", "ps_app_eval_shard_rows", "ps_shard_bounds", "ps_shard_step",
 ]
 # type-conversion methods for host inputs (Fig. 3)
 XFER_DEVICE, XFER_HOST_LOOP, XFER_HOST_SIMD, XFER_PIPELINE, XFER_TRANSIENT = 0, 1, 2, 3, 4
@@ -64,6 +64,15 @@ class PsResult(ctypes.Structure):
                 ("transfer_ms", ctypes.c_float), ("quality", ctypes.c_double),
                 ("max_rel", ctypes.c_double), ("nonfinite", ctypes.c_uint64),
                 ("pass_", ctypes.c_int32), ("status", ctypes.c_int32)]
+
+
+class PsShardRegion(ctypes.Structure):
+    _fields_ = [("ptr", ctypes.c_void_p), ("off", ctypes.c_uint64), ("len", ctypes.c_uint64)]
+
+
+class PsShardStep(ctypes.Structure):
+    _fields_ = [("done", ctypes.c_int32), ("nregions", ctypes.c_int32), ("region", PsShardRegion * 4),
+                ("result", PsResult)]
 
 
 class PsSearchResult(ctypes.Structure):
@@ -121,6 +130,11 @@ def lib():
                 "ps_app_reference_rows": (ctypes.c_int, [vp, ctypes.c_int64, ctypes.c_int64,
                                                          ctypes.POINTER(vp), vp]),
                 "ps_app_reference_merge": (ctypes.c_int, [vp, ctypes.POINTER(vp), vp]),
+                "ps_app_eval_shard_rows": (ctypes.c_int64, [vp]),
+                "ps_shard_bounds": (ctypes.c_int, [vp, ctypes.c_int, ctypes.c_int, i64p, i64p]),
+                "ps_shard_step": (ctypes.c_int, [vp, ctypes.POINTER(ctypes.c_int), ctypes.c_double,
+                                                 ctypes.c_int, ctypes.c_int, ctypes.c_int, vp,
+                                                 ctypes.POINTER(PsShardStep)]),
                 "ps_config_encode": (ctypes.c_int, [vp, ctypes.POINTER(ctypes.c_int),
                                                     ctypes.POINTER(ctypes.c_uint64)]),
                 "ps_config_decode": (ctypes.c_int, [vp, ctypes.c_uint64, ctypes.POINTER(ctypes.c_int)]),
@@ -352,6 +366,32 @@ class App:
         _check(lib().ps_app_reference_merge(self._h, arr, _stream(stream)), "ps_app_reference_merge")
         self.ref = list(refs)
         return refs
+
+    # ------------------------------------------- row-sharded evaluation (4b)
+    @property
+    def eval_shard_rows(self) -> int:
+        """Rows of the dimension a row-sharded evaluation splits (0: not supported)."""
+        return int(lib().ps_app_eval_shard_rows(self._h))
+
+    def shard_bounds(self, rank: int, world: int):
+        r0, r1 = ctypes.c_int64(), ctypes.c_int64()
+        _check(lib().ps_shard_bounds(self._h, int(rank), int(world), ctypes.byref(r0), ctypes.byref(r1)),
+               "ps_shard_bounds")
+        return int(r0.value), int(r1.value)
+
+    def shard_step(self, prec, rank: int, world: int, stage: int, toq: float = 0.9, stream=None):
+        """One stage of the row-sharded evaluation.  Returns (done, regions, result):
+        regions = [(workspace byte offset of the buffer, off, len)] to exchange, result
+        the record once done."""
+        p = (ctypes.c_int * self.num_objects)(*prec)
+        x = PsShardStep()
+        _check(lib().ps_shard_step(self._h, p, float(toq), int(rank), int(world), int(stage),
+                                   _stream(stream), ctypes.byref(x)), "ps_shard_step")
+        base = self.workspace.data_ptr()
+        regions = [(int(x.region[k].ptr) - base, int(x.region[k].off), int(x.region[k].len))
+                   for k in range(x.nregions)]
+        res = _result_dict(np.frombuffer(bytes(x.result), dtype=RESULT_DTYPE)[0]) if x.done else None
+        return bool(x.done), regions, res
 
     def set_reference(self, refs):
         arr = (vp * self.num_objects)(*[_ptr(t) for t in refs])

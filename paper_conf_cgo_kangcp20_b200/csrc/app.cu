@@ -21,6 +21,7 @@
 #include <atomic>
 #include <chrono>
 #include <map>
+#include <numeric>
 #include <mutex>
 #include <set>
 #include <thread>
@@ -228,6 +229,7 @@ struct ps_app {
   std::vector<cudaEvent_t> ev;
   QPart *host_res = nullptr;   // pinned, MAX_BATCH
   int device = -1;
+  float shard_ms[4] = {0, 0, 0, 0};   // ps_shard_step: a2 / a3 / a4+a5 / finalize, summed over stages
   ~ps_app() {
     for (auto e : ev) cudaEventDestroy(e);
     if (host_res) cudaFreeHost(host_res);
@@ -379,7 +381,9 @@ ps_status contraction(Ctx &c, GemmArgs g) {
   // E4M3/E5M2 in any mix, reading #29); f32 compute
   const bool pair = (g.A.type == g.B.type && (g.A.type == PS_F16 || g.A.type == PS_BF16)) ||
                     (is_fp8(g.A.type) && is_fp8(g.B.type));
-  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && pair && g.T == PS_F32 && g.row_off == 0 &&
+  // a row offset (sharded SYRK-like output) must keep the tile grid of the unsharded
+  // statement: both tcgen05 kernels then compute identical tiles
+  const bool tc = !(c.a->flags & PS_FLAG_NO_TENSOR_CORES) && pair && g.T == PS_F32 && g.row_off % 256 == 0 &&
                   gemm_tc_supported(g);
   if (!tc && (is_fp8(g.A.type) || is_fp8(g.B.type))) {
     set_error("internal: fp8 multiplicands reached the SIMT contraction");
@@ -408,6 +412,7 @@ GemmArgs matmul_args(Ctx &c, int x, int y, int out, int64_t M, int64_t N, int64_
   const int64_t r0 = rows && c.sharded() ? c.r0 : 0;
   GemmArgs g{};
   g.M = rows && c.sharded() ? c.r1 - c.r0 : M; g.N = N; g.K = K;
+  g.tc_m_full = M;
   g.A = MatDesc{eoff(c.ptr[x], c.prec[x], r0 * K), c.prec[x], K, 1, scale_of(c.a, x)};
   g.B = MatDesc{c.ptr[y], c.prec[y], N, 1, scale_of(c.a, y)};
   g.C = eoff(c.ptr[out], c.prec[out], r0 * N); g.c_type = c.prec[out]; g.ldc = N;
@@ -429,6 +434,7 @@ GemmArgs syrk_args(Ctx &c, int data, int sym, int64_t N, int64_t M, int epi, dou
   const int64_t r0 = c.sharded() ? c.r0 : 0;
   GemmArgs g{};
   g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
+  g.tc_m_full = M;
   g.A = MatDesc{eoff(c.ptr[data], c.prec[data], r0), c.prec[data], 1, M, scale_of(c.a, data)};   // A(j1, i) = data[i][j1]
   g.B = MatDesc{c.ptr[data], c.prec[data], M, 1, scale_of(c.a, data)};                          // B(i, j2) = data[i][j2]
   g.C = eoff(c.ptr[sym], c.prec[sym], r0 * M); g.c_type = c.prec[sym]; g.ldc = M;
@@ -459,6 +465,7 @@ GemmArgs gemm_args(Ctx &c) {   // C <- alpha (A.B) + beta C
   const int64_t r0 = c.sharded() ? c.r0 : 0;
   GemmArgs g{};
   g.M = c.sharded() ? c.r1 - c.r0 : d[0]; g.N = d[1]; g.K = d[2];
+  g.tc_m_full = d[0];
   g.A = MatDesc{eoff(c.ptr[0], c.prec[0], r0 * d[2]), c.prec[0], d[2], 1, scale_of(c.a, 0)};
   g.B = MatDesc{c.ptr[1], c.prec[1], d[1], 1, scale_of(c.a, 1)};
   g.C = eoff(c.ptr[2], c.prec[2], r0 * d[1]); g.c_type = c.prec[2]; g.ldc = d[1];
@@ -473,6 +480,7 @@ GemmArgs syr2k_args(Ctx &c, int s2) {   // C <- alpha X^T Y + beta C (s2 = 0: X=
   const int x = s2 ? 1 : 0, y = s2 ? 0 : 1;
   GemmArgs g{};
   g.M = c.sharded() ? c.r1 - c.r0 : M; g.N = M; g.K = N;
+  g.tc_m_full = M;
   g.A = MatDesc{eoff(c.ptr[x], c.prec[x], r0), c.prec[x], 1, M, scale_of(c.a, x)};   // A(i, k) = X[k][i]
   g.B = MatDesc{c.ptr[y], c.prec[y], M, 1, scale_of(c.a, y)};                       // B(k, j) = Y[k][j]
   g.C = eoff(c.ptr[2], c.prec[2], r0 * M); g.c_type = c.prec[2]; g.ldc = M;
@@ -599,8 +607,11 @@ ps_status run_statements(Ctx &c) {
     case K_SYRK:  // C <- alpha A^T A + beta C (upper tiles, mirrored)
       S_(syrk(c, 0, 1, d[0], d[1], EPI_AXPBY, 0.0, 0));
       break;
-    case K_CONV2D:
-      S_(stmt(c, OBJ(0), OBJ(1), [&] { return conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st); }));
+    case K_CONV2D:   // sharded: output rows [r0, r1) (ps_shard_step)
+      S_(stmt(c, OBJ(0), OBJ(1), [&] {
+        return c.sharded() ? conv2d_rows_async(P[0], p[0], P[1], p[1], d[0], d[1], c.r0, c.r1, c.st)
+                           : conv2d_async(P[0], p[0], P[1], p[1], d[0], d[1], c.st);
+      }));
       break;
     case K_SYR2K: {   // C <- alpha A^T B + beta C ; C <- alpha B^T A + C
       for (int s2 = 0; s2 < 2; s2++) {
@@ -612,8 +623,11 @@ ps_status run_statements(Ctx &c) {
       }
       break;
     }
-    case K_CONV3D:
-      S_(stmt(c, OBJ(0), OBJ(1), [&] { return conv3d_async(P[0], p[0], P[1], p[1], d[0], d[1], d[2], c.st); }));
+    case K_CONV3D:   // sharded: output planes [r0, r1)
+      S_(stmt(c, OBJ(0), OBJ(1), [&] {
+        return c.sharded() ? conv3d_rows_async(P[0], p[0], P[1], p[1], d[0], d[1], d[2], c.r0, c.r1, c.st)
+                           : conv3d_async(P[0], p[0], P[1], p[1], d[0], d[1], d[2], c.st);
+      }));
       break;
     case K_FDTD2D: {
       // statements per step (reading #27); with fp8 objects the ey row-0 assignment and
@@ -780,6 +794,441 @@ ps_status ready(const ps_app *a) {
   if (!a->bound) { set_error("app not bound (ps_app_bind)"); return PS_ERR_WORKSPACE; }
   if (!a->has_ref) { set_error("no reference (ps_app_reference)"); return PS_ERR_INVALID; }
   return PS_OK;
+}
+
+// ================================================ row-sharded evaluation (4b)
+// SURVEY §8(e) "very large objects: contiguous row-range shards".  One
+// configuration is evaluated by W ranks, each owning a contiguous range of the
+// app's sharded rows; the stages below exchange exactly what the statements need
+// (column-chunk partials, row blocks, quality segment partials) and every
+// reduction keeps its single-GPU association, so the record and the delivered
+// outputs are bit-identical to ps_run_config for every W.
+enum ShardProg { SP_NONE, SP_ATAX, SP_BICG, SP_GESUMMV, SP_MVT, SP_ROWS, SP_3MM, SP_SYRK, SP_CORR, SP_COVAR };
+
+struct ShardGeo {
+  int prog = SP_NONE;
+  int64_t rows = 0;    // the sharded dimension
+  int64_t align = 1;   // row bounds are multiples of this (except the last)
+  bool tri = false;    // balance on the cost of upper-triangular rows
+  int out = -1;        // the row-sharded scored output (-1: vector outputs, gathered)
+};
+
+ShardGeo shard_geo(const ps_app *a) {
+  ShardGeo g;
+  switch (a->kind) {
+    case K_ATAX: g.prog = SP_ATAX; break;
+    case K_BICG: g.prog = SP_BICG; break;
+    case K_GESUMMV: g.prog = SP_GESUMMV; break;
+    case K_MVT: g.prog = SP_MVT; break;
+    case K_GEMM: case K_2MM: case K_SYR2K: case K_CONV2D: case K_CONV3D: g.prog = SP_ROWS; break;
+    case K_3MM: g.prog = SP_3MM; break;
+    case K_SYRK: g.prog = SP_SYRK; break;
+    case K_CORR: g.prog = SP_CORR; break;
+    case K_COVAR: g.prog = SP_COVAR; break;
+    default: return g;   // FDTD-2D: TMAX dependent sweeps -- configurations are partitioned instead
+  }
+  if (g.prog == SP_ATAX || g.prog == SP_BICG || g.prog == SP_GESUMMV || g.prog == SP_MVT) {
+    g.rows = a->d[0];    // rows of A (and B)
+    g.align = g.prog == SP_GESUMMV ? 1 : COLSUM_CHUNK;
+    return g;
+  }
+  g.out = (a->kind == K_CONV2D || a->kind == K_CONV3D) ? 1 : shard_object(a);
+  g.rows = a->rows[g.out];
+  g.align = qseg(a->rows[g.out], a->cols[g.out]).rows_per;
+  if (a->kind != K_CONV2D && a->kind != K_CONV3D)   // contractions: whole 256-row tcgen05 tiles
+    g.align = std::lcm(g.align, (int64_t)256);
+  g.tri = a->kind == K_SYRK || a->kind == K_CORR || a->kind == K_COVAR;
+  return g;
+}
+
+// [r0, r1) of rank `rank` among `world`: contiguous, rounded to multiples of
+// `align`; tri balances sum_{i in range} (rows - i)
+void split_rows(int64_t rows, int world, int rank, int64_t align, bool tri, int64_t *r0, int64_t *r1) {
+  auto cut = [&](int r) -> int64_t {
+    if (r <= 0) return 0;
+    if (r >= world) return rows;
+    double b;
+    if (!tri) {
+      b = (double)rows * r / world;
+    } else {   // b rows cost b*rows - b(b-1)/2 = target
+      const double R = (double)rows, T = R * (R + 1) / 2.0 * r / world, q = 2 * R + 1;
+      b = (q - sqrt(q * q - 8 * T)) / 2;
+    }
+    int64_t v = (int64_t)llround(b / (double)align) * align;
+    return v < 0 ? 0 : (v > rows ? rows : v);
+  };
+  *r0 = cut(rank);
+  *r1 = std::max(*r0, cut(rank + 1));
+}
+
+Ctx shard_ctx(ps_app *a, const int *prec, cudaStream_t st) {
+  Ctx c{a, {0}, {nullptr}, st};
+  for (int m = 0; m < a->def->nobj; m++) {
+    c.prec[m] = prec[m];
+    c.ptr[m] = (a->def->o[m].role == 0 && prec[m] == PS_F32) ? (void *)a->orig_in[m] : a->ws + a->slot_off[m];
+  }
+  return c;
+}
+
+// a2 for rows [r0, r1) of an input / inout object (r1 < 0: every row)
+ps_status a2_rows(ps_app *a, Ctx &c, int m, int64_t r0 = 0, int64_t r1 = -1) {
+  const int role = a->def->o[m].role;
+  if (role != 0 && role != 2) return PS_OK;
+  if (role == 0 && c.prec[m] == PS_F32) return PS_OK;   // used in place
+  if (r1 < 0) r1 = a->rows[m];
+  r0 = std::max<int64_t>(r0, 0);
+  r1 = std::min<int64_t>(r1, a->rows[m]);
+  if (r1 <= r0) return PS_OK;
+  const int64_t cols = a->cols[m];
+  return convert_async(a->orig_in[m] + r0 * cols, PS_F32, eoff(c.ptr[m], c.prec[m], r0 * cols), c.prec[m],
+                       (size_t)((r1 - r0) * cols), c.st);
+}
+
+ps_shard_region row_region(ps_app *a, Ctx &c, int m, int64_t r0, int64_t r1) {
+  const uint64_t rb = (uint64_t)a->cols[m] * dtype_size(c.prec[m]);
+  return ps_shard_region{c.ptr[m], (uint64_t)r0 * rb, (uint64_t)(r1 - r0) * rb};
+}
+
+// column-chunk partials of a rows-of-A shard: T-typed [nchunks][cols] at the
+// workspace partial area; the shard's chunks start at chunk r0 / COLSUM_CHUNK
+void *spart_at(ps_app *a, int T, int64_t r0, int64_t cols) {
+  return a->ws + a->partial_off + (size_t)(r0 / COLSUM_CHUNK) * (size_t)cols * dtype_size(T);
+}
+void *qpart_of(ps_app *a, int64_t rows, int64_t cols) {
+  return a->ws + a->partial_off + tile_spart_bytes(rows, cols);
+}
+ps_shard_region spart_region(ps_app *a, int T, int64_t r0, int64_t r1, int64_t cols) {
+  const uint64_t cb = (uint64_t)cols * dtype_size(T);
+  const uint64_t c0 = (uint64_t)(r0 / COLSUM_CHUNK), c1 = (uint64_t)((r1 + COLSUM_CHUNK - 1) / COLSUM_CHUNK);
+  return ps_shard_region{a->ws + a->partial_off, c0 * cb, (c1 > c0 ? c1 - c0 : 0) * cb};
+}
+
+// a4 + a5 of every output over its full extent (vector outputs, present on every rank)
+ps_status quality_all(ps_app *a, Ctx &c, QPart *res) {
+  QPart *parts = (QPart *)(a->ws + a->qparts_off);
+  int np = 0;
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!a->def->o[m].is_output) continue;
+    PS_TRY(backconv_quality_async(c.ptr[m], c.prec[m], a->ref[m], a->orig_out[m], a->rows[m], a->cols[m],
+                                  parts + np, c.st));
+    np += qseg(a->rows[m], a->cols[m]).nb;
+  }
+  return quality_finalize_async(parts, np, res, c.st);
+}
+
+// a4 + a5 partials of rows [r0, r1) of the row-sharded output m (whole segments)
+ps_status quality_rows(ps_app *a, Ctx &c, int m, int64_t r0, int64_t r1, ps_shard_region *reg) {
+  QPart *parts = (QPart *)(a->ws + a->qparts_off);
+  const QSeg q = qseg(a->rows[m], a->cols[m]);
+  const int s0 = (int)(r0 / q.rows_per);
+  const int s1 = r1 >= a->rows[m] ? q.nb : (int)(r1 / q.rows_per);
+  *reg = ps_shard_region{parts, (uint64_t)s0 * sizeof(QPart), (uint64_t)(s1 > s0 ? s1 - s0 : 0) * sizeof(QPart)};
+  if (s1 <= s0) return PS_OK;
+  return backconv_quality_async(c.ptr[m], c.prec[m], a->ref[m], a->orig_out[m], a->rows[m], a->cols[m], parts,
+                                c.st, s0, s1);
+}
+ps_status quality_rows_finalize(ps_app *a, int m, QPart *res, cudaStream_t st) {
+  return quality_finalize_async((QPart *)(a->ws + a->qparts_off), qseg(a->rows[m], a->cols[m]).nb, res, st);
+}
+
+// One stage of the program; events ev[0..4] bracket a2 / statements / a4+a5 partials /
+// finalize (as enqueue_config); *done when res holds the final quality.
+ps_status shard_stage(ps_app *a, const int *prec, int rank, int world, int stage, cudaStream_t st,
+                      cudaEvent_t *ev, QPart *res, ps_shard_step_t *x) {
+  const ShardGeo g = shard_geo(a);
+  const int64_t *d = a->d;
+  Ctx c = shard_ctx(a, prec, st);
+  const int *p = c.prec;
+  void **P = c.ptr;
+  int64_t r0, r1;
+  split_rows(g.rows, world, rank, g.align, g.tri, &r0, &r1);
+  x->done = 0;
+  x->nregions = 0;
+  auto region = [&](ps_shard_region r) { x->region[x->nregions++] = r; };
+  auto rec = [&](int k) -> ps_status {
+    PS_CUDA(cudaEventRecord(ev[k], st));
+    return PS_OK;
+  };
+  const int last_rec = 4;
+  (void)last_rec;
+  switch (g.prog) {
+    // ------------------------------------------------------------ mat-vec apps
+    case SP_ATAX: {   // tmp <- A x (rows) ; y <- A^T tmp (chunk partials -> gather -> finalize)
+      const int T2 = compute_type({p[0], p[3], p[2]});
+      if (stage == 0) {
+        PS_TRY(rec(0));
+        PS_TRY(a2_rows(a, c, 0, r0, r1));
+        PS_TRY(a2_rows(a, c, 1));
+        PS_TRY(rec(1));
+        if (r1 > r0) {
+          PS_TRY(tile_rows_async(-1, eoff(P[0], p[0], r0 * d[1]), p[0], d[1], nullptr, PS_F32, P[1], p[1],
+                                 eoff(P[3], p[3], r0), p[3], 0, r1 - r0, d[1], PS_F32, nullptr,
+                                 qpart_of(a, d[0], d[1]), st));
+          PS_TRY(tile_rows_async(COL_DOT, eoff(P[0], p[0], r0 * d[1]), p[0], d[1], eoff(P[3], p[3], r0), p[3],
+                                 nullptr, PS_F32, nullptr, PS_F32, 0, r1 - r0, d[1], T2, spart_at(a, T2, r0, d[1]),
+                                 qpart_of(a, d[0], d[1]), st));
+        }
+        PS_TRY(rec(2));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(spart_region(a, T2, r0, r1, d[1]));
+        return PS_OK;
+      }
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(colsum_finalize_async(a->ws + a->partial_off, T2, d[0], d[1], P[2], p[2], FIN_PLAIN, 0, 0, st));
+      PS_TRY(rec(2));
+      PS_TRY(quality_all(a, c, res));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      x->done = 1;
+      return PS_OK;
+    }
+    case SP_BICG: {   // s <- A^T r (chunk partials) ; q <- A p (rows) -- one pass over the rows
+      const int T1 = compute_type({p[0], p[1], p[2]});
+      if (stage == 0) {
+        PS_TRY(rec(0));
+        PS_TRY(a2_rows(a, c, 0, r0, r1));
+        PS_TRY(a2_rows(a, c, 1));
+        PS_TRY(a2_rows(a, c, 3));
+        PS_TRY(rec(1));
+        if (r1 > r0)
+          PS_TRY(tile_rows_async(COL_DOT, eoff(P[0], p[0], r0 * d[1]), p[0], d[1], eoff(P[1], p[1], r0), p[1],
+                                 P[3], p[3], eoff(P[4], p[4], r0), p[4], 0, r1 - r0, d[1], T1,
+                                 spart_at(a, T1, r0, d[1]), qpart_of(a, d[0], d[1]), st));
+        PS_TRY(rec(2));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(spart_region(a, T1, r0, r1, d[1]));
+        region(row_region(a, c, 4, r0, r1));   // q: a vector, "rows" = elements
+        return PS_OK;
+      }
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(colsum_finalize_async(a->ws + a->partial_off, T1, d[0], d[1], P[2], p[2], FIN_PLAIN, 0, 0, st));
+      PS_TRY(rec(2));
+      PS_TRY(quality_all(a, c, res));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      x->done = 1;
+      return PS_OK;
+    }
+    case SP_GESUMMV: {   // tmp, y rows of A x, B x; y <- alpha tmp + beta y (rows); gather y
+      if (stage == 0) {
+        PS_TRY(rec(0));
+        PS_TRY(a2_rows(a, c, 0, r0, r1));
+        PS_TRY(a2_rows(a, c, 1, r0, r1));
+        PS_TRY(a2_rows(a, c, 2));
+        PS_TRY(rec(1));
+        if (r1 > r0) {
+          PS_TRY(tile_rows_async(-1, eoff(P[0], p[0], r0 * d[0]), p[0], d[0], nullptr, PS_F32, P[2], p[2],
+                                 eoff(P[4], p[4], r0), p[4], 0, r1 - r0, d[0], PS_F32, nullptr,
+                                 qpart_of(a, d[0], d[0]), st));
+          PS_TRY(tile_rows_async(-1, eoff(P[1], p[1], r0 * d[0]), p[1], d[0], nullptr, PS_F32, P[2], p[2],
+                                 eoff(P[3], p[3], r0), p[3], 0, r1 - r0, d[0], PS_F32, nullptr,
+                                 qpart_of(a, d[0], d[0]), st));
+          PS_TRY(axpby_async(eoff(P[4], p[4], r0), p[4], eoff(P[3], p[3], r0), p[3], r1 - r0, a->sc[0], a->sc[1],
+                             st));
+        }
+        PS_TRY(rec(2));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(row_region(a, c, 3, r0, r1));
+        return PS_OK;
+      }
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(rec(2));
+      PS_TRY(quality_all(a, c, res));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      x->done = 1;
+      return PS_OK;
+    }
+    case SP_MVT: {   // x1 <- x1 + A y1 (rows) ; x2 <- x2 + A^T y2 (chunk partials)
+      const int TC = compute_type({p[0], p[2], p[4]});
+      if (stage == 0) {
+        PS_TRY(rec(0));
+        PS_TRY(a2_rows(a, c, 0, r0, r1));
+        for (int m = 1; m < 5; m++) PS_TRY(a2_rows(a, c, m));
+        PS_TRY(rec(1));
+        if (r1 > r0)
+          PS_TRY(tile_rows_async(COL_DOT, eoff(P[0], p[0], r0 * d[0]), p[0], d[0], eoff(P[4], p[4], r0), p[4],
+                                 P[3], p[3], eoff(P[1], p[1], r0), p[1], 1, r1 - r0, d[0], TC,
+                                 spart_at(a, TC, r0, d[0]), qpart_of(a, d[0], d[0]), st));
+        PS_TRY(rec(2));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(row_region(a, c, 1, r0, r1));
+        region(spart_region(a, TC, r0, r1, d[0]));
+        return PS_OK;
+      }
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(colsum_finalize_async(a->ws + a->partial_off, TC, d[0], d[0], P[2], p[2], FIN_ADD, 0, 0, st));
+      PS_TRY(rec(2));
+      PS_TRY(quality_all(a, c, res));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      x->done = 1;
+      return PS_OK;
+    }
+    // ------------------------------------------- row-local contractions / stencils
+    case SP_ROWS: {   // GEMM, 2MM, SYR2K, 2DCONV, 3DCONV: rows of the output need no exchange
+      if (stage == 0) {
+        PS_TRY(rec(0));
+        switch (a->kind) {
+          case K_GEMM: PS_TRY(a2_rows(a, c, 0, r0, r1)); PS_TRY(a2_rows(a, c, 1)); PS_TRY(a2_rows(a, c, 2, r0, r1)); break;
+          case K_2MM: PS_TRY(a2_rows(a, c, 0, r0, r1)); PS_TRY(a2_rows(a, c, 1)); PS_TRY(a2_rows(a, c, 3)); break;
+          case K_SYR2K: PS_TRY(a2_rows(a, c, 0)); PS_TRY(a2_rows(a, c, 1)); PS_TRY(a2_rows(a, c, 2, r0, r1)); break;
+          default: PS_TRY(a2_rows(a, c, 0, r0 - 1, r1 + 1)); break;   // stencils: + one-row halo
+        }
+        PS_TRY(rec(1));
+        c.r0 = r0;
+        c.r1 = r1;
+        if (r1 > r0) PS_TRY(run_statements(c));
+        PS_TRY(rec(2));
+        ps_shard_region q;
+        PS_TRY(quality_rows(a, c, g.out, r0, r1, &q));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(q);
+        return PS_OK;
+      }
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(rec(2));
+      PS_TRY(rec(3));
+      PS_TRY(quality_rows_finalize(a, g.out, res, st));
+      PS_TRY(rec(4));
+      x->done = 1;
+      return PS_OK;
+    }
+    case SP_3MM: {   // E rows (A rows) and F rows (own split) ; gather F ; G rows ; quality
+      int64_t f0, f1;
+      split_rows(d[1], world, rank, 256, false, &f0, &f1);
+      if (stage == 0) {
+        PS_TRY(rec(0));
+        PS_TRY(a2_rows(a, c, 0, r0, r1));
+        PS_TRY(a2_rows(a, c, 1));
+        PS_TRY(a2_rows(a, c, 2, f0, f1));
+        PS_TRY(a2_rows(a, c, 3));
+        PS_TRY(rec(1));
+        c.r0 = r0;
+        c.r1 = r1;
+        if (r1 > r0) PS_TRY(matmul(c, 0, 1, 4, d[0], d[1], d[2], true));   // E <- A.B
+        c.r0 = f0;
+        c.r1 = f1;
+        if (f1 > f0) PS_TRY(matmul(c, 2, 3, 5, d[1], d[3], d[4], true));   // F <- C.D (rows f0..f1)
+        PS_TRY(rec(2));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(row_region(a, c, 5, f0, f1));
+        return PS_OK;
+      }
+      if (stage == 1) {
+        PS_TRY(rec(0));
+        PS_TRY(rec(1));
+        c.r0 = r0;
+        c.r1 = r1;
+        if (r1 > r0) PS_TRY(matmul(c, 4, 5, 6, d[0], d[3], d[1], true));   // G <- E.F
+        PS_TRY(rec(2));
+        ps_shard_region q;
+        PS_TRY(quality_rows(a, c, 6, r0, r1, &q));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(q);
+        return PS_OK;
+      }
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(rec(2));
+      PS_TRY(rec(3));
+      PS_TRY(quality_rows_finalize(a, 6, res, st));
+      PS_TRY(rec(4));
+      x->done = 1;
+      return PS_OK;
+    }
+    // ---------------------------------------------- symmetric outputs (upper + mirror)
+    case SP_SYRK:
+    case SP_CORR:
+    case SP_COVAR: {
+      const int sym = g.out;
+      const int data_stages = g.prog == SP_SYRK ? 0 : (g.prog == SP_CORR ? 3 : 2);
+      const int64_t N = d[0], M = d[1];
+      int64_t d0, d1;   // data rows (CORR / COVAR column statistics)
+      split_rows(N, world, rank, COLSUM_CHUNK, false, &d0, &d1);
+      const int T1 = compute_type({p[0], p[1]});                                  // mean
+      const int T2 = g.prog == SP_CORR ? compute_type({p[0], p[1], p[2]}) : T1;    // stddev / normalise
+      PS_TRY(rec(0));
+      if (stage == 0 && g.prog != SP_SYRK) {   // a2 of the data rows, mean partials
+        PS_TRY(a2_rows(a, c, 0, d0, d1));
+        PS_TRY(rec(1));
+        if (d1 > d0)
+          PS_TRY(tile_rows_async(COL_SUM, eoff(P[0], p[0], d0 * M), p[0], M, nullptr, PS_F32, nullptr, PS_F32,
+                                 nullptr, PS_F32, 0, d1 - d0, M, T1, spart_at(a, T1, d0, M), qpart_of(a, N, M), st));
+        region(spart_region(a, T1, d0, d1, M));
+      } else if (stage == 1 && g.prog == SP_CORR) {   // mean; stddev partials
+        PS_TRY(rec(1));
+        PS_TRY(colsum_finalize_async(a->ws + a->partial_off, T1, N, M, P[1], p[1], FIN_MEAN, (double)N, 0, st));
+        if (d1 > d0)
+          PS_TRY(tile_rows_async(COL_SQDEV, eoff(P[0], p[0], d0 * M), p[0], M, P[1], p[1], nullptr, PS_F32,
+                                 nullptr, PS_F32, 0, d1 - d0, M, T2, spart_at(a, T2, d0, M), qpart_of(a, N, M), st));
+        region(spart_region(a, T2, d0, d1, M));
+      } else if (stage == data_stages - 1 && g.prog != SP_SYRK) {   // finish stats, normalise rows
+        PS_TRY(rec(1));
+        if (g.prog == SP_CORR) {
+          PS_TRY(colsum_finalize_async(a->ws + a->partial_off, T2, N, M, P[2], p[2], FIN_STDDEV, (double)N,
+                                       a->sc[0], st));
+          if (d1 > d0)
+            PS_TRY(corr_normalize_async(eoff(P[0], p[0], d0 * M), p[0], P[1], p[1], P[2], p[2], d1 - d0, M,
+                                        sqrt((double)N), st));
+        } else {
+          PS_TRY(colsum_finalize_async(a->ws + a->partial_off, T1, N, M, P[1], p[1], FIN_MEAN, (double)N, 0, st));
+          if (d1 > d0) PS_TRY(covar_center_async(eoff(P[0], p[0], d0 * M), p[0], P[1], p[1], d1 - d0, M, st));
+        }
+        region(row_region(a, c, 0, d0, d1));
+      } else if (stage == data_stages) {   // upper part of the output rows
+        if (g.prog == SP_SYRK) {
+          PS_TRY(a2_rows(a, c, 0));
+          PS_TRY(a2_rows(a, c, 1, r0, r1));
+        }
+        PS_TRY(rec(1));
+        c.r0 = r0;
+        c.r1 = r1;
+        if (r1 > r0) {
+          if (g.prog == SP_SYRK) PS_TRY(syrk(c, 0, 1, N, M, EPI_AXPBY, 0.0, 0));
+          else if (g.prog == SP_CORR) PS_TRY(syrk(c, 0, 3, N, M, EPI_PLAIN, 0.0, 1));
+          else PS_TRY(syrk(c, 0, 2, N, M, EPI_DIV, (double)N - 1.0, 0));
+        }
+        region(row_region(a, c, sym, r0, r1));
+      } else if (stage == data_stages + 1) {   // mirror, quality partials of the rows
+        PS_TRY(rec(1));
+        PS_TRY(mirror_async(P[sym], p[sym], M, g.prog == SP_CORR ? 1 : 0, st));
+        PS_TRY(rec(2));
+        ps_shard_region q;
+        PS_TRY(quality_rows(a, c, sym, r0, r1, &q));
+        PS_TRY(rec(3));
+        PS_TRY(rec(4));
+        region(q);
+        return PS_OK;
+      } else {
+        PS_TRY(rec(1));
+        PS_TRY(rec(2));
+        PS_TRY(rec(3));
+        PS_TRY(quality_rows_finalize(a, sym, res, st));
+        PS_TRY(rec(4));
+        x->done = 1;
+        return PS_OK;
+      }
+      PS_TRY(rec(2));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      return PS_OK;
+    }
+  }
+  set_error("ps_shard_step: %s has no row-sharded evaluation", a->def->kind);
+  return PS_ERR_UNSUPPORTED;
 }
 
 }  // namespace
@@ -1280,6 +1729,57 @@ ps_status ps_search(ps_app *a, double toq, int repeats, void *stream, ps_search_
   out->total_ms = tcur.ms;
   out->quality = tcur.q;
   out->pass = tcur.pass;
+  return PS_OK;
+}
+
+int64_t ps_app_eval_shard_rows(const ps_app *a) { return a ? shard_geo(a).rows : 0; }
+
+ps_status ps_shard_bounds(const ps_app *a, int rank, int world, int64_t *row0, int64_t *row1) {
+  if (!a || !row0 || !row1 || world < 1 || rank < 0 || rank >= world) {
+    set_error("ps_shard_bounds: bad argument");
+    return PS_ERR_INVALID;
+  }
+  const ShardGeo g = shard_geo(a);
+  if (!g.rows) { set_error("ps_shard_bounds: %s has no row-sharded evaluation", a->def->kind); return PS_ERR_UNSUPPORTED; }
+  split_rows(g.rows, world, rank, g.align, g.tri, row0, row1);
+  return PS_OK;
+}
+
+ps_status ps_shard_step(ps_app *a, const int *prec, double toq, int rank, int world, int stage, void *stream,
+                        ps_shard_step_t *x) {
+  ps_status s = ready(a);
+  if (s != PS_OK) return s;
+  if (!x || world < 1 || rank < 0 || rank >= world || stage < 0) {
+    set_error("ps_shard_step: bad argument");
+    return PS_ERR_INVALID;
+  }
+  if ((s = check_prec(a, prec)) != PS_OK) return s;
+  for (int m = 0; m < a->def->nobj; m++)
+    if (is_fp8(prec[m])) {   // a per-tensor scale needs the amax of the whole object
+      set_error("ps_shard_step: fp8 objects are not row-shardable (per-tensor scale)");
+      return PS_ERR_UNSUPPORTED;
+    }
+  if (!shard_geo(a).rows) { set_error("ps_shard_step: %s has no row-sharded evaluation", a->def->kind); return PS_ERR_UNSUPPORTED; }
+  if ((s = ensure_events(a, NEV)) != PS_OK) return s;
+  cudaStream_t st = (cudaStream_t)stream;
+  if (stage == 0) memset(a->shard_ms, 0, sizeof(a->shard_ms));
+  QPart *res = (QPart *)(a->ws + a->qres_off);
+  memset(x, 0, sizeof(*x));
+  s = shard_stage(a, prec, rank, world, stage, st, a->ev.data(), res, x);
+  if (s != PS_OK) return s;
+  if (x->done) PS_CUDA(cudaMemcpyAsync(a->host_res, res, sizeof(QPart), cudaMemcpyDeviceToHost, st));
+  PS_CUDA(cudaStreamSynchronize(st));
+  for (int k = 0; k < 4; k++) a->shard_ms[k] += ms_between(a->ev[k], a->ev[k + 1]);
+  if (x->done) {
+    uint64_t id = 0;
+    ps_config_encode(a, prec, &id);
+    fill_result(a, id, a->host_res[0], a->ev.data(), toq, &x->result);
+    x->result.convert_ms = a->shard_ms[0];
+    x->result.kernel_ms = a->shard_ms[1];
+    x->result.backconv_ms = a->shard_ms[2];
+    x->result.quality_ms = a->shard_ms[3];
+    x->result.total_ms = a->shard_ms[0] + a->shard_ms[1] + a->shard_ms[2];
+  }
   return PS_OK;
 }
 

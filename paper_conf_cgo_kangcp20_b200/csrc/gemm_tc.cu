@@ -70,6 +70,7 @@ struct Params {
   int epi;
   float alpha, beta, div;
   int upper_only;
+  int row_off;             // upper_only: global row of output row 0 (row-sharded evaluation)
   uint32_t a_fmt, b_fmt;   // kind::f16: 0 = f16, 1 = bf16 (reading #28); kind::f8f6f4: 0 = E4M3, 1 = E5M2
   const ps_fp8_scale *sa, *sb;   // fp8 operands: per-tensor scales (reading #29)
   int vec4;                // C / Cin rows 4-element aligned: vector epilogue stores / loads
@@ -284,7 +285,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
-  if (p.upper_only && m0 >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
+  if (p.upper_only && m0 + p.row_off >= n0 + BN) return;   // SYRK: tile strictly below the diagonal
   const int nk = (p.K + BK - 1) / BK;
 
   if (warp == 0 && lane == 0) {
@@ -470,11 +471,12 @@ __device__ __forceinline__ void arrive_leader(uint64_t *bar) {
 struct Sched {
   int64_t tiles_m, tiles_n, total;
   int upper_only;
+  int64_t tm_off;          // upper_only: global tile row of tile row 0 (row_off / BM)
   // i-th tile of this cluster (skipping SYRK lower tiles); false when exhausted
   __device__ bool get(int64_t cluster, int64_t nclusters, int64_t &cursor, int &m0, int &n0) const {
     for (int64_t t = cursor; t < total; t += nclusters) {
       const int64_t tm = t / tiles_n, tn = t % tiles_n;
-      if (upper_only && tm > tn) continue;
+      if (upper_only && tm + tm_off > tn) continue;
       m0 = (int)(tm * BM);
       n0 = (int)(tn * BN);
       cursor = t + nclusters;
@@ -693,7 +695,10 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   CUtensorMap ma, mb;
   const bool a_mn = !(g.A.s_col == 1);
   const bool b_k = !(g.B.s_col == 1);
-  const bool two = (g.M > BM || g.N > BN) && !getenv("PS_TC_1SM");
+  // the kernel choice follows the unsharded shape (tc_m_full) so that every shard of
+  // a row-sharded evaluation runs the same tiles as the single-GPU statement
+  const int64_t m_shape = g.tc_m_full > 0 ? g.tc_m_full : g.M;
+  const bool two = (m_shape > BM || g.N > BN) && !getenv("PS_TC_1SM");
   bool ok;
   if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * ES, BM, g.A.type);
   else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * ES, G::BK, g.A.type);
@@ -707,7 +712,7 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   const uint32_t af = (g.A.type == PS_BF16 || g.A.type == PS_E5M2) ? 1u : 0u;
   const uint32_t bfm = (g.B.type == PS_BF16 || g.B.type == PS_E5M2) ? 1u : 0u;
   Params p{(int)g.M, (int)g.N, (int)g.K, a_mn ? 1 : 0, b_k ? 1 : 0, g.C, g.c_type, g.ldc, g.Cin, g.cin_type, g.epi,
-           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, af, bfm,
+           (float)g.alpha, (float)g.beta, (float)g.div, g.upper_only, (int)g.row_off, af, bfm,
            ES == 1 ? g.A.sc : nullptr, ES == 1 ? g.B.sc : nullptr, 0};
   {   // vector epilogue: rows of C (and Cin) start 16-byte (f32) / 8-byte (16-bit) aligned
     const int64_t cb = (int64_t)dtype_size(g.c_type);
@@ -723,9 +728,10 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
     sch.tiles_n = (g.N + tc2::BN - 1) / tc2::BN;
     sch.total = sch.tiles_m * sch.tiles_n;
     sch.upper_only = g.upper_only;
+    sch.tm_off = g.row_off / tc2::BM;
     int64_t work = 0;
     for (int64_t t = 0; t < sch.total; t++)
-      if (!g.upper_only || t / sch.tiles_n <= t % sch.tiles_n) work++;
+      if (!g.upper_only || t / sch.tiles_n + sch.tm_off <= t % sch.tiles_n) work++;
     int64_t clusters = num_sms() / 2;
     if (clusters > work) clusters = work;
     if (clusters < 1) clusters = 1;

@@ -59,7 +59,8 @@ struct GemmArgs {
   int epi;
   double alpha, beta, div;   // fp64 literals (rounded to T on the device side)
   int upper_only;       // SYRK: skip tiles strictly below the diagonal
-  int64_t row_off;      // upper_only: global index of row 0 of C (row-sharded reference)
+  int64_t row_off;      // upper_only: global index of row 0 of C (row-sharded reference / evaluation)
+  int64_t tc_m_full;    // > 0: M of the unsharded statement (tcgen05 picks its kernel from it)
   int T;                // compute type PS_F32 / PS_F64
 };
 // R3-exact SIMT contraction (FFMA / DFMA fma chains, k ascending)
@@ -91,9 +92,13 @@ ps_status mvt_async(const void *A, int ta, int64_t n, void *x1, int t1, void *x2
                     const void *y1, int ty1, const void *y2, int ty2, void *partial, cudaStream_t st);
 // 2DCONV 3x3 stencil (reading #24): B_ij = sum of 9 rounded products, left to right; border +0
 ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, cudaStream_t st);
+ps_status conv2d_rows_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t ibeg,
+                            int64_t iend, cudaStream_t st);   // output rows [ibeg, iend)
 // 3DCONV 27-point stencil (reading #26) on NI x NJ x NK
 ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
                        cudaStream_t st);
+ps_status conv3d_rows_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
+                            int64_t ibeg, int64_t iend, cudaStream_t st);   // output planes [ibeg, iend)
 // one statement of FDTD-2D time step t (reading #27): FDTD_EY = ey row 0 from fict and
 // the ey update in one pass; FDTD_EY0 / FDTD_EY1 = those two parts alone (reading #29)
 enum FdtdPart { FDTD_EY = 0, FDTD_EY0 = 1, FDTD_EY1 = 2, FDTD_EX = 3, FDTD_HZ = 4 };
@@ -102,6 +107,15 @@ ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int te
 ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
                        int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
                        double eps, void *partial, cudaStream_t st);
+// row-sharded pieces (tiles.cu): one rank's tile pass over its rows (column-chunk
+// partials into the full array at `spart`, row dots finished locally), and the
+// in-order finalize over every chunk; mode COL_* or -1 (row dots only)
+ps_status tile_rows_async(int mode, const void *A, int ta, int64_t lda, const void *w, int tw,
+                          const void *x, int tx, void *rd_out, int t_rd, int rd_add, int64_t rows,
+                          int64_t cols, int TC, void *spart, void *qpart, cudaStream_t st);
+ps_status colsum_finalize_async(const void *spart, int TC, int64_t rows, int64_t cols, void *out, int tout,
+                                int fin, double n, double eps, cudaStream_t st);
+size_t tile_spart_bytes(int64_t rows, int64_t cols);   // the full chunk-partial array (8-byte entries)
 // y_i = RNE_y(fma(alpha, tmp_i, beta * y_i)) in T = W(tmp, y)
 ps_status axpby_async(const void *tmp, int ttmp, void *y, int ty, int64_t n, double alpha,
                       double beta, cudaStream_t st);

@@ -24,14 +24,15 @@ template <class T> struct Coef9 { T c[9]; };
 template <class SA, class SB>
 __global__ void __launch_bounds__(NT) conv2d_kernel(const raw_t<SA> *__restrict__ A,
                                                     raw_t<SB> *__restrict__ B, int64_t ni,
-                                                    int64_t nj, Coef9<T2<SA, SB>> cf, int vec_ok) {
+                                                    int64_t nj, Coef9<T2<SA, SB>> cf, int vec_ok,
+                                                    int64_t ibeg, int64_t iend) {
   using T = T2<SA, SB>;
   using RA = raw_t<SA>;
   constexpr int V = 16 / (int)sizeof(RA);          // elements per 16-byte vector
   // staged window: rows i0-1 .. i0+TY, cols j0-V .. j0+TX+V-1 (16-byte aligned)
   constexpr int HW = TX + 2 * V, HH = TY + 2, NV = HW / V, HN = NV * HH;
   __shared__ T tile[HH][HW];
-  const int64_t i0 = (int64_t)blockIdx.y * TY, j0 = (int64_t)blockIdx.x * TX;
+  const int64_t i0 = ibeg + (int64_t)blockIdx.y * TY, j0 = (int64_t)blockIdx.x * TX;
   const bool inner = vec_ok && i0 >= 1 && j0 >= V && i0 + TY + 1 <= ni && j0 + TX + V <= nj;
   constexpr int PER = (HN + NT - 1) / NT;
   union Vec { uint4 u; RA e[V]; } v[PER];
@@ -66,7 +67,7 @@ __global__ void __launch_bounds__(NT) conv2d_kernel(const raw_t<SA> *__restrict_
 #pragma unroll 4
   for (int r = 0; r < RY; r++) {
     const int64_t i = i0 + ty0 + r;
-    if (i >= ni) break;
+    if (i >= iend) break;
     T acc = T(0);
     if (i > 0 && j > 0 && i + 1 < ni && j + 1 < nj) {
       // (di, dj) in the order c11, c12, c13, c21, c22, c23, c31, c32, c33
@@ -81,10 +82,13 @@ __global__ void __launch_bounds__(NT) conv2d_kernel(const raw_t<SA> *__restrict_
   }
 }
 
-ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, cudaStream_t st) {
-  if (ni <= 0 || nj <= 0) return PS_OK;
+// output rows [ibeg, iend) of the full NI x NJ problem (borders by the global
+// indices); the rows read are [ibeg - 1, iend + 1) -- a row-sharded evaluation
+ps_status conv2d_rows_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t ibeg,
+                            int64_t iend, cudaStream_t st) {
+  if (ni <= 0 || nj <= 0 || iend <= ibeg) return PS_OK;
   static const double C[9] = {0.2, -0.3, 0.4, 0.5, 0.6, 0.7, -0.8, -0.9, 0.10};
-  dim3 grid((unsigned)((nj + TX - 1) / TX), (unsigned)((ni + TY - 1) / TY));
+  dim3 grid((unsigned)((nj + TX - 1) / TX), (unsigned)((iend - ibeg + TY - 1) / TY));
   return dispatch_store(ta, [&](auto sa) -> ps_status {
     return dispatch_store(tb, [&](auto sb) -> ps_status {
       using SA = decltype(sa);
@@ -93,11 +97,16 @@ ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64
       Coef9<T> cf;
       for (int k = 0; k < 9; k++) cf.c[k] = (T)C[k];   // RNE from the fp64 literal (R2)
       const int vec_ok = ((uintptr_t)A % 16 == 0) && ((nj * (int64_t)sizeof(raw_t<SA>)) % 16 == 0);
-      conv2d_kernel<SA, SB><<<grid, NT, 0, st>>>((const raw_t<SA> *)A, (raw_t<SB> *)B, ni, nj, cf, vec_ok);
+      conv2d_kernel<SA, SB><<<grid, NT, 0, st>>>((const raw_t<SA> *)A, (raw_t<SB> *)B, ni, nj, cf, vec_ok,
+                                                 ibeg, iend);
       PS_CHECK_LAUNCH("conv2d_kernel");
       return PS_OK;
     });
   });
+}
+
+ps_status conv2d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, cudaStream_t st) {
+  return conv2d_rows_async(A, ta, B, tb, ni, nj, 0, ni, st);
 }
 
 // ------------------------------------------------------------------- 3DCONV
@@ -135,7 +144,7 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 template <class SA, class SB>
 __global__ void __launch_bounds__(C3_NT, sizeof(T2<SA, SB>) == 8 ? 2 : 3) conv3d_kernel(
     const raw_t<SA> *__restrict__ A, raw_t<SB> *__restrict__ B, int64_t ni, int64_t nj, int64_t nk,
-    Coef27<T2<SA, SB>> cf, int vec_ok) {
+    Coef27<T2<SA, SB>> cf, int vec_ok, int64_t ibeg, int64_t iend) {
   using T = T2<SA, SB>;
   using RA = raw_t<SA>;
   using G = C3Geo<SA>;
@@ -147,8 +156,8 @@ __global__ void __launch_bounds__(C3_NT, sizeof(T2<SA, SB>) == 8 ? 2 : 3) conv3d
   T(*sl)[C3_SH][SW] = reinterpret_cast<T(*)[C3_SH][SW]>(c3_smem);
   RA(*rw)[C3_SH][SW] = reinterpret_cast<RA(*)[C3_SH][SW]>(c3_smem + sizeof(T) * C3_RING * C3_SH * SW);
   const int64_t k0 = (int64_t)blockIdx.x * C3_TK, j0 = (int64_t)blockIdx.y * C3_TJ;
-  const int64_t ib = (int64_t)blockIdx.z * C3_IL;
-  const int64_t ie = ib + C3_IL < ni ? ib + C3_IL : ni;       // output planes [ib, ie)
+  const int64_t ib = ibeg + (int64_t)blockIdx.z * C3_IL;
+  const int64_t ie = ib + C3_IL < iend ? ib + C3_IL : iend;   // output planes [ib, ie)
   const int64_t plane = nj * nk;
   int64_t off[PER];                                            // window element offsets in a slice
   bool in[PER];                                                // vector inside the (j, k) range
@@ -286,13 +295,14 @@ __global__ void __launch_bounds__(C3_NT, sizeof(T2<SA, SB>) == 8 ? 2 : 3) conv3d
   }
 }
 
-ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
-                       cudaStream_t st) {
-  if (ni <= 0 || nj <= 0 || nk <= 0) return PS_OK;
+// output planes [ibeg, iend) (planes [ibeg - 1, iend + 1) are read): row-sharded evaluation
+ps_status conv3d_rows_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
+                            int64_t ibeg, int64_t iend, cudaStream_t st) {
+  if (ni <= 0 || nj <= 0 || nk <= 0 || iend <= ibeg) return PS_OK;
   static const double C[9] = {0.2, -0.3, 0.4, 0.5, 0.6, 0.7, -0.8, -0.9, 0.10};
   static const double G[3] = {0.25, 0.5, 0.25};
   dim3 grid((unsigned)((nk + C3_TK - 1) / C3_TK), (unsigned)((nj + C3_TJ - 1) / C3_TJ),
-            (unsigned)((ni + C3_IL - 1) / C3_IL));
+            (unsigned)((iend - ibeg + C3_IL - 1) / C3_IL));
   return dispatch_store(ta, [&](auto sa) -> ps_status {
     return dispatch_store(tb, [&](auto sb) -> ps_status {
       using SA = decltype(sa);
@@ -306,11 +316,16 @@ ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64
       const int vec_ok = ((uintptr_t)A % 16 == 0) && ((nk * (int64_t)sizeof(raw_t<SA>)) % 16 == 0);
       PS_TRY(set_max_smem((const void *)conv3d_kernel<SA, SB>, (int)smem));
       conv3d_kernel<SA, SB><<<grid, C3_NT, smem, st>>>((const raw_t<SA> *)A, (raw_t<SB> *)B, ni, nj, nk, cf,
-                                                         vec_ok);
+                                                         vec_ok, ibeg, iend);
       PS_CHECK_LAUNCH("conv3d_kernel");
       return PS_OK;
     });
   });
+}
+
+ps_status conv3d_async(const void *A, int ta, void *B, int tb, int64_t ni, int64_t nj, int64_t nk,
+                       cudaStream_t st) {
+  return conv3d_rows_async(A, ta, B, tb, ni, nj, nk, 0, ni, st);
 }
 
 // ------------------------------------------------------------------ FDTD-2D

@@ -413,4 +413,55 @@ ps_status bicg_async(const void *A, int ta, int64_t lda, const void *r, int tr, 
   return TR == PS_F64 ? rowdot_finalize<double>(a, q, tq, st) : rowdot_finalize<float>(a, q, tq, st);
 }
 
+// ------------------------------------------------ row-sharded pieces (ps_shard_step)
+// One rank's tile pass over its rows of A: A, w (COL_DOT weights) and the row-dot
+// output start at the rank's first row r0 (a multiple of COLSUM_CHUNK), `spart`
+// points at chunk r0 / COLSUM_CHUNK of the FULL column-chunk partial array (typed
+// TC, cols per chunk), so every rank fills its own chunks of the same array; row
+// dots (rd_out != nullptr) are finished locally for the rank's rows.  After the
+// chunks of all ranks are in place, colsum_finalize_async adds them in chunk order
+// -- the same association as the unsharded statement (R5), so the result is
+// bit-identical for any rank count.
+ps_status tile_rows_async(int mode, const void *A, int ta, int64_t lda, const void *w, int tw,
+                          const void *x, int tx, void *rd_out, int t_rd, int rd_add, int64_t rows,
+                          int64_t cols, int TC, void *spart, void *qpart, cudaStream_t st) {
+  if (rows <= 0 || cols <= 0) return PS_OK;
+  TileArgs a = make_args(A, ta, lda, rows, cols, nullptr);
+  a.spart = spart;
+  a.qpart = qpart;
+  a.w = w;
+  a.tw = w ? tw : PS_F32;
+  a.x = x;
+  a.tx = x ? tx : PS_F32;
+  const bool rd = rd_out != nullptr;
+  const int TR = rd ? compute_type({ta, tx, t_rd}) : TC;
+  ps_status e;
+  if (rd && mode == CM_NONE) e = tile_dispatch<CM_NONE, true>(a, ta, TR, TR, st);
+  else if (rd && mode == COL_DOT) e = tile_dispatch<COL_DOT, true>(a, ta, TC, TR, st);
+  else if (!rd && mode == COL_DOT) e = tile_dispatch<COL_DOT, false>(a, ta, TC, TC, st);
+  else if (!rd && mode == COL_SUM) e = tile_dispatch<COL_SUM, false>(a, ta, TC, TC, st);
+  else if (!rd && mode == COL_SQDEV) e = tile_dispatch<COL_SQDEV, false>(a, ta, TC, TC, st);
+  else {
+    set_error("tile_rows_async: unsupported mode");
+    return PS_ERR_UNSUPPORTED;
+  }
+  if (e != PS_OK || !rd) return e;
+  return TR == PS_F64 ? rowdot_finalize<double>(a, rd_out, t_rd, st, rd_add)
+                      : rowdot_finalize<float>(a, rd_out, t_rd, st, rd_add);
+}
+
+ps_status colsum_finalize_async(const void *spart, int TC, int64_t rows, int64_t cols, void *out, int tout,
+                                int fin, double n, double eps, cudaStream_t st) {
+  if (rows <= 0 || cols <= 0) return PS_OK;
+  TileArgs a{};
+  a.spart = const_cast<void *>(spart);
+  a.rows = rows;
+  a.cols = cols;
+  a.nchunks = nchunks_of(rows);
+  return TC == PS_F64 ? colsum_finalize<double>(a, out, tout, fin, n, eps, st)
+                      : colsum_finalize<float>(a, out, tout, fin, n, eps, st);
+}
+
+size_t tile_spart_bytes(int64_t rows, int64_t cols) { return spart_bytes(rows, cols); }
+
 }  // namespace ps

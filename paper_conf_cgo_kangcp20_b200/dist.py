@@ -225,3 +225,52 @@ def sharded_reference(app, world: int, rank: int, group=None, refs=None):
 def env_rank():
     return (int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)),
             int(os.environ.get("LOCAL_RANK", 0)))
+
+
+# ------------------------------------------- row-sharded evaluation of ONE config
+def exchange_regions(workspace, regions, group=None):
+    """All-gather the byte ranges each rank produced in a shard stage: rank r owns
+    [off_r, off_r + len_r) of the buffer at workspace offset `base` (same on every
+    rank); afterwards every rank holds every rank's range.  One all_gather of the
+    (base, off, len) triples, then per region one all_gather_into_tensor of the
+    pieces padded to the longest (NCCL over NVLink; gloo in the CPU tests)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    dev = workspace.device
+    k = len(regions)
+    meta = torch.tensor([v for r in regions for v in r] or [0], dtype=torch.int64, device=dev)
+    allm = torch.zeros(world * meta.numel(), dtype=torch.int64, device=dev)
+    dist.all_gather_into_tensor(allm, meta, group=group)
+    allm = allm.view(world, -1).cpu().tolist()
+    for j in range(k):
+        spans = [(allm[q][3 * j], allm[q][3 * j + 1], allm[q][3 * j + 2]) for q in range(world)]
+        mx = max(s[2] for s in spans)
+        if mx == 0:
+            continue
+        base, off, ln = spans[rank]
+        send = torch.zeros(mx, dtype=torch.uint8, device=dev)
+        send[:ln] = workspace[base + off:base + off + ln]
+        recv = torch.empty(world * mx, dtype=torch.uint8, device=dev)
+        dist.all_gather_into_tensor(recv, send, group=group)
+        for q, (b, o, n) in enumerate(spans):
+            if q != rank and n:
+                workspace[b + o:b + o + n] = recv[q * mx:q * mx + n]
+
+
+def sharded_evaluate(app, prec, toq: float = 0.9, group=None, stream=None):
+    """ONE configuration evaluated by every rank of the group, each on its
+    contiguous row range (ps_shard_step + exchange_regions); returns the record,
+    identical on every rank and bit-identical to app.run_config(prec)."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    stage = 0
+    while True:
+        done, regions, res = app.shard_step(prec, rank, world, stage, toq, stream)
+        if done:
+            return res
+        if world > 1:
+            exchange_regions(app.workspace, regions, group)
+        stage += 1

@@ -148,3 +148,42 @@ def test_gather_rows_world2_gloo(kind, dims):
     for _, raw in out:
         got = np.frombuffer(raw, dtype=np.float64)
         assert got.tobytes() == np.ascontiguousarray(ref[m], dtype=np.float64).reshape(-1).tobytes()
+
+
+# ------------------------------------------- row-sharded evaluation exchange
+def _xchg_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ws = torch.zeros(4096, dtype=torch.uint8)
+    # two regions at workspace offsets 100 and 2000; rank r owns uneven (possibly empty) ranges
+    spans = [[(0, 37), (37, 37), (37, 300)], [(0, 8), (8, 24), (24, 1000)]]
+    regions = []
+    for j, base in enumerate((100, 2000)):
+        o0, o1 = spans[j][rank]
+        ws[base + o0:base + o1] = torch.arange(o0, o1, dtype=torch.int64).to(torch.uint8) + 7 * j + 1
+        regions.append((base, o0, o1 - o0))
+    D.exchange_regions(ws, regions)
+    q.put((rank, ws.numpy().tobytes()))
+    dist.destroy_process_group()
+
+
+def test_exchange_regions_world3_gloo():
+    """dist.exchange_regions (the NCCL all-gather of ps_shard_step's byte ranges):
+    every rank ends with every rank's range, including empty ones."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_xchg_worker, args=(r, 3, port, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    out = sorted(q.get(timeout=120) for _ in range(3))
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    want = np.zeros(4096, dtype=np.uint8)
+    want[100:400] = (np.arange(300) + 1).astype(np.uint8)
+    want[2000:3000] = (np.arange(1000) + 8).astype(np.uint8)
+    for _, raw in out:
+        assert np.frombuffer(raw, dtype=np.uint8).tobytes() == want.tobytes()
