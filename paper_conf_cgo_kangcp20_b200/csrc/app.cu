@@ -888,6 +888,11 @@ ps_shard_region row_region(ps_app *a, Ctx &c, int m, int64_t r0, int64_t r1) {
   const uint64_t rb = (uint64_t)a->cols[m] * dtype_size(c.prec[m]);
   return ps_shard_region{c.ptr[m], (uint64_t)r0 * rb, (uint64_t)(r1 - r0) * rb};
 }
+// elements [e0, e1) of a vector object (the row-dot outputs of the mat-vec apps)
+ps_shard_region vec_region(Ctx &c, int m, int64_t e0, int64_t e1) {
+  const uint64_t es = dtype_size(c.prec[m]);
+  return ps_shard_region{c.ptr[m], (uint64_t)e0 * es, (uint64_t)(e1 - e0) * es};
+}
 
 // column-chunk partials of a rows-of-A shard: T-typed [nchunks][cols] at the
 // workspace partial area; the shard's chunks start at chunk r0 / COLSUM_CHUNK
@@ -1000,7 +1005,8 @@ ps_status shard_stage(ps_app *a, const int *prec, int rank, int world, int stage
         PS_TRY(rec(3));
         PS_TRY(rec(4));
         region(spart_region(a, T1, r0, r1, d[1]));
-        region(row_region(a, c, 4, r0, r1));   // q: a vector, "rows" = elements
+        region(vec_region(c, 4, r0, r1));       // q
+
         return PS_OK;
       }
       PS_TRY(rec(0));
@@ -1033,7 +1039,7 @@ ps_status shard_stage(ps_app *a, const int *prec, int rank, int world, int stage
         PS_TRY(rec(2));
         PS_TRY(rec(3));
         PS_TRY(rec(4));
-        region(row_region(a, c, 3, r0, r1));
+        region(vec_region(c, 3, r0, r1));       // y
         return PS_OK;
       }
       PS_TRY(rec(0));
@@ -1059,7 +1065,7 @@ ps_status shard_stage(ps_app *a, const int *prec, int rank, int world, int stage
         PS_TRY(rec(2));
         PS_TRY(rec(3));
         PS_TRY(rec(4));
-        region(row_region(a, c, 1, r0, r1));
+        region(vec_region(c, 1, r0, r1));       // x1
         region(spart_region(a, TC, r0, r1, d[0]));
         return PS_OK;
       }
