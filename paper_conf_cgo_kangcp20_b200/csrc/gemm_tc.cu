@@ -24,6 +24,8 @@
 // elements wide; the epilogue multiplies the f32 accumulator by the operands'
 // per-tensor scales 2^(ka + kb) (exact) before alpha/beta.
 #include <cuda.h>
+
+#include <atomic>
 #include <cudaTypedefs.h>
 
 #include "common.cuh"
@@ -39,13 +41,15 @@ constexpr int B_BYTES = BN * KB_BYTES;          // 32 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 // epilogue staging: each of the 4 epilogue warps turns a 32 x 32 accumulator chunk
 // (thread = row, from tcgen05.ld.32x32b) into coalesced row segments through smem
-constexpr int EPI_COLS = 32;
-constexpr int EPI_STRIDE = 36;                                // floats per staged row (conflict-free float4)
+// 16-column chunks (round 2: from 32) halve the staging buffer, which buys the 2-CTA
+// kernel a sixth pipeline stage
+constexpr int EPI_COLS = 16;
+constexpr int EPI_STRIDE = 20;                                // floats per staged row (conflict-free STS.128)
 // 8 epilogue warps: two per TMEM lane quarter (warp w may read lanes 32 (w % 4)..),
 // each draining half of the accumulator's columns -- twice the memory-level
 // parallelism of one warp per quarter, which paced the fp8 tiles (ncu, round 1)
 constexpr int EPI_WARPS = 8;
-constexpr int EPI_SMEM = EPI_WARPS * 32 * EPI_STRIDE * 4;     // 36 KiB
+constexpr int EPI_SMEM = EPI_WARPS * 32 * EPI_STRIDE * 4;     // 20 KiB
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + EPI_SMEM;
 constexpr int NTHREADS = 64 + 32 * EPI_WARPS;
 constexpr uint32_t TMEM_COLS = 256;
@@ -192,28 +196,29 @@ __device__ __forceinline__ float epi_op(const Params &p, float r, float cin) {
   return r;
 }
 
-// Epilogue of one 32-row x 32-column accumulator chunk held by this warp (lane =
-// row row0 + lane, v = columns col0..col0+31 from tcgen05.ld.32x32b.x32): staged
-// through smem, then written as coalesced row segments -- lane l handles row
-// 4i + l/8 and columns 4(l%8)..+3 (one 16-byte f32 or 8-byte 16-bit access, and
-// the matching Cin load for alpha/beta).  fp8 operands: accumulator x 2^kab first.
+// Epilogue of one 32-row x 16-column accumulator chunk held by this warp (lane =
+// row row0 + lane, v = columns col0..col0+15 from tcgen05.ld.32x32b.x16): staged
+// through smem, then written as row segments -- lane l handles rows 8i + l/4 and
+// columns 4(l%4)..+3 (one 16-byte f32 or 8-byte 16-bit access, and the matching
+// Cin load for alpha/beta), so 4 lanes cover a row's 64 contiguous bytes.  fp8
+// operands: accumulator x 2^kab first.
 __device__ __forceinline__ void epi_chunk(const Params &p, float *stg, int lane, int64_t row0,
-                                          int64_t col0, const uint32_t (&v)[32], int kab) {
+                                          int64_t col0, const uint32_t (&v)[16], int kab) {
   float4 *srow = reinterpret_cast<float4 *>(stg + lane * EPI_STRIDE);
 #pragma unroll
-  for (int q = 0; q < 8; q++)
+  for (int q = 0; q < 4; q++)
     srow[q] = make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]),
                           __uint_as_float(v[4 * q + 2]), __uint_as_float(v[4 * q + 3]));
   __syncwarp();
-  const int cq = lane & 7;
+  const int cq = lane & 3;
   const int64_t col = col0 + cq * 4;
   const bool vcol = p.vec4 && col + 3 < p.N;
-  // 1) the chunk's 8 Cin segments of this lane, all loads in flight at once (alpha/beta)
-  float c[8][4];
+  // 1) the chunk's 4 Cin segments of this lane, all loads in flight at once (alpha/beta)
+  float c[4][4];
 #pragma unroll
-  for (int i = 0; i < 8; i++) {
+  for (int i = 0; i < 4; i++) {
     c[i][0] = c[i][1] = c[i][2] = c[i][3] = 0.f;
-    const int64_t row = row0 + i * 4 + (lane >> 3);
+    const int64_t row = row0 + i * 8 + (lane >> 2);
     if (p.epi != EPI_AXPBY || row >= p.M) continue;
     const int64_t idx = row * p.ldc + col;
     if (vcol) {
@@ -233,10 +238,10 @@ __device__ __forceinline__ void epi_chunk(const Params &p, float *stg, int lane,
         if (col + e < p.N) c[i][e] = load_c(p.Cin, p.cin_type, idx + e);
     }
   }
-  // 2) scale, epilogue op, RNE store (R1) as coalesced row segments
+  // 2) scale, epilogue op, RNE store (R1) as row segments
 #pragma unroll
-  for (int i = 0; i < 8; i++) {
-    const int r = i * 4 + (lane >> 3);
+  for (int i = 0; i < 4; i++) {
+    const int r = i * 8 + (lane >> 2);
     const int64_t row = row0 + r;
     const float4 a = *reinterpret_cast<const float4 *>(stg + r * EPI_STRIDE + cq * 4);
     float x[4] = {a.x, a.y, a.z, a.w};
@@ -371,8 +376,8 @@ __global__ void __launch_bounds__(NTHREADS, 1)
     const int half = (warp - 2) / 4;        // which half of the columns this warp drains
     for (int cc = half * (BN / EPI_COLS / 2); cc < (half + 1) * (BN / EPI_COLS / 2); cc++) {
       if ((int64_t)n0 + cc * EPI_COLS >= p.N) break;
-      uint32_t v[32];
-      tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
+      uint32_t v[16];
+      tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
       epi_chunk(p, stg, lane, (int64_t)m0 + q * 32, (int64_t)n0 + cc * EPI_COLS, v, kab);
     }
   }
@@ -395,7 +400,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 // c, c + #clusters, ... (SYRK: lower tiles skipped by every role alike).
 namespace tc2 {
 
-constexpr int BM = 256, BN = 256, STAGES = 5;
+constexpr int BM = 256, BN = 256, STAGES = 6;   // 6 x 32 KiB + 20 KiB epilogue staging
 constexpr int HM = BM / 2, HN = BN / 2;          // per-CTA halves
 constexpr int A_BYTES = HM * tc::KB_BYTES;      // 16 KiB
 constexpr int B_BYTES = HN * tc::KB_BYTES;      // 16 KiB
@@ -416,6 +421,7 @@ using tc::mbar_wait;
 using tc::smem_u32;
 using tc::tmem_ld16;
 using tc::tmem_ld32;
+using tc::tmem_ld16;
 using tc::epi_chunk;
 using tc::EPI_COLS;
 using tc::EPI_STRIDE;
@@ -438,6 +444,16 @@ __device__ __forceinline__ void tma_load_2sm(void *dst, const CUtensorMap *map, 
       "l"((uint64_t)map), "r"(smem_u32(bar) & PEER_MASK), "r"(c0), "r"(c1)
       : "memory");
 }
+// multicast variant: the box lands at the same smem offset in every CTA of `mask`;
+// each destination's bytes complete on ITS pair leader's barrier (peer bit cleared)
+__device__ __forceinline__ void tma_load_2sm_mc(void *dst, const CUtensorMap *map, uint64_t *bar, int c0, int c1,
+                                                uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+      " [%0], [%1, {%4, %5}], [%2], %3;" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)map), "r"(smem_u32(bar) & PEER_MASK), "h"(mask), "r"(c0), "r"(c1)
+      : "memory");
+}
 template <int ES>
 __device__ __forceinline__ void umma2(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   const uint32_t z = 0;
@@ -454,31 +470,41 @@ __device__ __forceinline__ void umma2(uint32_t tmem_d, uint64_t a, uint64_t b, u
         "tcgen05.mma.cta_group::2.kind::f8f6f4 [%0], %1, %2, %3, {%5, %5, %5, %5, %5, %5, %5, %5}, p;\n\t}" ::"r"(tmem_d),
         "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(z));
 }
-__device__ __forceinline__ void commit_both(uint64_t *bar) {
+// commit the leader's MMAs to the barrier at this offset in every CTA of `mask`
+__device__ __forceinline__ void commit_mc(uint64_t *bar, uint16_t mask) {
   asm volatile(
       "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
           smem_u32(bar)),
-      "h"((uint16_t)3)
+      "h"(mask)
       : "memory");
 }
-// arrive on the leader CTA's copy of a barrier (remote for rank 1)
-__device__ __forceinline__ void arrive_leader(uint64_t *bar) {
+// arrive on the pair leader's copy of a barrier (remote for odd ranks)
+__device__ __forceinline__ void arrive_leader(uint64_t *bar, uint32_t leader_rank) {
   uint32_t remote;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(remote) : "r"(smem_u32(bar)));
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(smem_u32(bar)), "r"(leader_rank));
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(remote) : "memory");
 }
 
 struct Sched {
-  int64_t tiles_m, tiles_n, total;
+  int64_t tiles_m, tiles_n, total;   // tiles_n counts cluster tiles of npairs * BN columns
+  int npairs;                        // CTA pairs per cluster (1, or 2 with A multicast)
   int upper_only;
   int64_t tm_off;          // upper_only: global tile row of tile row 0 (row_off / BM)
-  // i-th tile of this cluster (skipping SYRK lower tiles); false when exhausted
+  // i-th tile of this cluster (skipping SYRK tiles wholly below the diagonal); n0 is the
+  // cluster tile's first column -- pair p computes columns n0 + p * BN ..
+  // Grouped raster: consecutive t walk GROUP_M tile-rows down a tile-column before
+  // moving right, so the ~74 tiles in flight share ~8 A row-blocks and ~10 B column
+  // blocks (~70 MB at K = 8192 fp16) that stay in L2, instead of one tile-row
+  // against all of B (round-2 ncu: 2.3 GB DRAM reads per 8192^3 GEMM, L2 hit 65%).
+  static constexpr int64_t GROUP_M = 8;
   __device__ bool get(int64_t cluster, int64_t nclusters, int64_t &cursor, int &m0, int &n0) const {
     for (int64_t t = cursor; t < total; t += nclusters) {
-      const int64_t tm = t / tiles_n, tn = t % tiles_n;
-      if (upper_only && tm + tm_off > tn) continue;
+      const int64_t per_group = GROUP_M * tiles_n, g = t / per_group, first = g * GROUP_M;
+      const int64_t gm = tiles_m - first < GROUP_M ? tiles_m - first : GROUP_M;
+      const int64_t tm = first + (t % per_group) % gm, tn = (t % per_group) / gm;
+      if (upper_only && tm + tm_off > tn * npairs + npairs - 1) continue;
       m0 = (int)(tm * BM);
-      n0 = (int)(tn * BN);
+      n0 = (int)(tn * BN * npairs);
       cursor = t + nclusters;
       return true;
     }
@@ -487,8 +513,13 @@ struct Sched {
   }
 };
 
-template <int ES>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
+// CL = 2: one CTA pair per cluster.  CL = 4: two pairs side by side along N
+// (a 256 x 512 cluster tile) sharing the A rows -- each CTA loads half of its A
+// block (64 rows) and multicasts it to the same-rank CTA of the other pair, so a
+// CTA reads 24 KiB instead of 32 KiB from L2 per k-block; a stage is free once
+// BOTH pairs' MMAs retired it (empty barrier count 2, commits multicast to all 4).
+template <int ES, int CL>
+__global__ void __launch_bounds__(NTHREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
                     Params p, Sched sch) {
   using G = Geo<ES>;
@@ -505,9 +536,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
   float *epi_stage = (float *)(smem + STAGES * STAGE_BYTES + 512);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t rank = cluster_rank();
+  const uint32_t crank = cluster_rank();
+  const uint32_t rank = crank & 1u, pair = crank >> 1;   // rank within the pair, pair in the cluster
   const bool leader = rank == 0;
-  const int64_t cluster = blockIdx.x >> 1, nclusters = gridDim.x >> 1;
+  const uint16_t pair_mask = (uint16_t)(3u << (2 * pair));
+  const int64_t cluster = blockIdx.x / CL, nclusters = gridDim.x / CL;
   const int nk = (p.K + BK - 1) / BK;
 
   if (warp == 0 && lane == 0) {
@@ -515,11 +548,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tma_b) : "memory");
     for (int s = 0; s < STAGES; s++) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], 1);
+      mbar_init(&empty[s], CL / 2);   // every pair leader's commit (A is shared across pairs)
     }
     for (int a = 0; a < 2; a++) {
       mbar_init(&tfull[a], 1);
-      mbar_init(&tempty[a], 2 * tc::EPI_WARPS);   // every epilogue warp of both CTAs
+      mbar_init(&tempty[a], 2 * tc::EPI_WARPS);   // every epilogue warp of both CTAs of the pair
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -539,7 +572,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
       int m0, n0;
       uint32_t it = 0;
       while (sch.get(cluster, nclusters, cursor, m0, n0)) {
-        const int am = m0 + (int)rank * HM, bn = n0 + (int)rank * HN;
+        const int am = m0 + (int)rank * HM, bn = n0 + (int)pair * BN + (int)rank * HN;
         for (int kb = 0; kb < nk; kb++, it++) {
           const int s = it % STAGES;
           const uint32_t ph = (it / STAGES) & 1u;
@@ -547,7 +580,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
           if (leader) mbar_expect_tx(&full[s], 2 * STAGE_BYTES);   // both CTAs' bytes
           const int k0 = kb * BK;
           uint8_t *a = sA + s * A_BYTES;
-          if (!p.a_mn_major) {
+          if constexpr (CL == 4) {   // my half of the A block, to me and my counterpart
+            const uint16_t amask = (uint16_t)((1u << rank) | (1u << (rank + 2)));
+            if (!p.a_mn_major)                                              // box {BK, 64 M}
+              tma_load_2sm_mc(a + pair * (HM / 2) * tc::KB_BYTES, &tma_a, &full[s], k0,
+                              am + (int)pair * (HM / 2), amask);
+            else                                                            // box {MN_BOX M, BK}
+              tma_load_2sm_mc(a + pair * G::BOX_BYTES, &tma_a, &full[s], am + G::MN_BOX * (int)pair, k0, amask);
+          } else if (!p.a_mn_major) {
             tma_load_2sm(a, &tma_a, &full[s], k0, am);                    // box {BK, 128 M}
           } else {
 #pragma unroll
@@ -591,9 +631,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
                                             : umma_desc(bbase + kk * G::MN_STEP, G::BOX_BYTES, 1024);
             umma2<ES>(dcol, ad, bd, idesc, (kb | kk) != 0);
           }
-          commit_both(&empty[s]);   // stage s free in both CTAs once these MMAs retire
+          // stage s free once these MMAs retire: both CTAs of the pair, and with A
+          // multicast the other pair too (its producers write into our stage)
+          commit_mc(&empty[s], CL == 4 ? (uint16_t)0xF : pair_mask);
         }
-        commit_both(&tfull[acc]);   // accumulator acc complete in both CTAs
+        commit_mc(&tfull[acc], pair_mask);   // accumulator acc complete in both CTAs of the pair
         j++;
       }
     }
@@ -608,17 +650,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NTHREADS, 1)
       mbar_wait(&tfull[acc], (j >> 1) & 1u);
       fence_after();
       const int64_t row0 = (int64_t)m0 + rank * HM + q * 32;
+      const int64_t pn0 = (int64_t)n0 + pair * BN;
       float *stg = epi_stage + (warp - 2) * 32 * EPI_STRIDE;
       const int half = (warp - 2) / 4;
       for (int cc = half * (BN / EPI_COLS / 2); cc < (half + 1) * (BN / EPI_COLS / 2); cc++) {
-        if ((int64_t)n0 + cc * EPI_COLS >= p.N) break;
-        uint32_t v[32];
-        tmem_ld32(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
-        epi_chunk(p, stg, lane, row0, (int64_t)n0 + cc * EPI_COLS, v, kab);
+        if (pn0 + cc * EPI_COLS >= p.N) break;
+        uint32_t v[16];
+        tmem_ld16(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
+        epi_chunk(p, stg, lane, row0, pn0 + cc * EPI_COLS, v, kab);
       }
       fence_before();
       __syncwarp();
-      if (lane == 0) arrive_leader(&tempty[acc]);
+      if (lane == 0) arrive_leader(&tempty[acc], crank & ~1u);
       j++;
     }
   }
@@ -699,8 +742,16 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
   // a row-sharded evaluation runs the same tiles as the single-GPU statement
   const int64_t m_shape = g.tc_m_full > 0 ? g.tc_m_full : g.M;
   const bool two = (m_shape > BM || g.N > BN) && !getenv("PS_TC_1SM");
+  // two CTA pairs per cluster sharing A (multicast) when a row of tiles has >= 2 pair tiles;
+  // f16 / bf16 only (an fp8 M-major A box is the whole 128-row half)
+  // Tried in round 2: clusters of two CTA pairs sharing A by TMA multicast (a CTA reads
+  // 24 instead of 32 KiB per k-block).  Correct, but only 33 four-CTA clusters are
+  // co-resident on a B200 (GPC shape; ncu launch__cluster_max_active), i.e. 132 of 148
+  // SMs: 1329 vs 1363 TFLOP/s fp16 at 8192^3 (profiles/kernel_rates_r2g.jsonl).  Off.
+  const bool four = false;
   bool ok;
-  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * ES, BM, g.A.type);
+  if (!a_mn) ok = make_map(&ma, g.A.p, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.A.s_row * ES,
+                           four ? tc2::HM / 2 : BM, g.A.type);
   else ok = make_map(&ma, g.A.p, (uint64_t)g.M, (uint64_t)g.K, (uint64_t)g.A.s_col * ES, G::BK, g.A.type);
   if (!b_k) ok = ok && make_map(&mb, g.B.p, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.B.s_row * ES, G::BK, g.B.type);
   else ok = ok && make_map(&mb, g.B.p, (uint64_t)g.K, (uint64_t)g.N, (uint64_t)g.B.s_col * ES,
@@ -720,22 +771,48 @@ static ps_status gemm_tc_launch(const GemmArgs &g, cudaStream_t st) {
     if (g.epi == EPI_AXPBY) v4 = v4 && (uintptr_t)g.Cin % (4 * dtype_size(g.cin_type)) == 0;
     p.vec4 = v4 ? 1 : 0;
   }
-  if (two) {   // 2-CTA persistent path
+  if (two) {   // 2-CTA persistent path (clusters of 1 or 2 CTA pairs)
     using namespace tc2;
-    PS_TRY(set_max_smem((const void *)gemm_tc2_kernel<ES>, tc2::SMEM_BYTES));
+    const int CL = four ? 4 : 2;
+    const void *kfn = four ? (const void *)gemm_tc2_kernel<ES, 4> : (const void *)gemm_tc2_kernel<ES, 2>;
+    PS_TRY(set_max_smem(kfn, tc2::SMEM_BYTES));
     Sched sch;
+    sch.npairs = CL / 2;
     sch.tiles_m = (g.M + tc2::BM - 1) / tc2::BM;
-    sch.tiles_n = (g.N + tc2::BN - 1) / tc2::BN;
+    sch.tiles_n = (g.N + tc2::BN * sch.npairs - 1) / (tc2::BN * sch.npairs);
     sch.total = sch.tiles_m * sch.tiles_n;
     sch.upper_only = g.upper_only;
     sch.tm_off = g.row_off / tc2::BM;
     int64_t work = 0;
     for (int64_t t = 0; t < sch.total; t++)
-      if (!g.upper_only || t / sch.tiles_n + sch.tm_off <= t % sch.tiles_n) work++;
-    int64_t clusters = num_sms() / 2;
+      if (!g.upper_only || t / sch.tiles_n + sch.tm_off <= (t % sch.tiles_n) * sch.npairs + sch.npairs - 1) work++;
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)CL;
+    attr[0].val.clusterDim.y = attr[0].val.clusterDim.z = 1;
+    cfg.blockDim = dim3(tc2::NTHREADS);
+    cfg.dynamicSmemBytes = tc2::SMEM_BYTES;
+    cfg.stream = st;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    // persistent: no more clusters than can be co-resident (4-CTA clusters must fit a GPC)
+    int64_t clusters = num_sms() / CL;
+    {
+      static std::atomic<int> resident[2] = {0, 0};
+      int r = resident[CL == 4].load(std::memory_order_relaxed);
+      if (!r) {
+        cfg.gridDim = dim3((unsigned)(CL * clusters));
+        if (cudaOccupancyMaxActiveClusters(&r, kfn, &cfg) != cudaSuccess || r < 1) r = (int)clusters;
+        resident[CL == 4].store(r, std::memory_order_relaxed);
+      }
+      if (clusters > r) clusters = r;
+    }
     if (clusters > work) clusters = work;
     if (clusters < 1) clusters = 1;
-    gemm_tc2_kernel<ES><<<(unsigned)(2 * clusters), tc2::NTHREADS, tc2::SMEM_BYTES, st>>>(ma, mb, p, sch);
+    cfg.gridDim = dim3((unsigned)(CL * clusters));
+    if (four) PS_CUDA(cudaLaunchKernelEx(&cfg, gemm_tc2_kernel<ES, 4>, ma, mb, p, sch));
+    else PS_CUDA(cudaLaunchKernelEx(&cfg, gemm_tc2_kernel<ES, 2>, ma, mb, p, sch));
     PS_CHECK_LAUNCH("gemm_tc2_kernel");
     return PS_OK;
   }

@@ -12,7 +12,12 @@ KEYS = ["gpu__time_duration.sum", "launch__registers_per_thread", "launch__grid_
         "dram__bytes_read.sum", "dram__bytes_write.sum",
         "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
         "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum",
-        "lts__t_sector_hit_rate.pct"]
+        "lts__t_sector_hit_rate.pct",
+        "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+        "sm__mem_tensor_cycles_active.avg.pct_of_peak_sustained_active",
+        "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+        "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed"]
 
 
 def summarise(path, source):
@@ -24,6 +29,11 @@ def summarise(path, source):
     for k in KEYS:
         if k in d:
             out[k] = "%s %s" % (d[k], u.get(k, ""))
+        else:   # section-prefixed names (e.g. "TPC.TriageCompute.<metric>")
+            for kk in d:
+                if kk.endswith("." + k):
+                    out[k] = "%s %s" % (d[kk], u.get(kk, ""))
+                    break
     stalls = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): float(v.replace(",", ""))
               for k, v in d.items() if k.startswith("smsp__pcsamp_warps_issue_stalled_")
               and not k.endswith("not_issued") and v.replace(",", "").replace(".", "").isdigit()}
