@@ -703,34 +703,50 @@ def main():
         d2h = sum(len(a["ids"]) * 24 for a in apps)      # one (sum e, max, count) record per config
 
         copy = torch.cuda.Stream()
+        # two device input sets per app: step k sweeps set k % 2 while step k+1's inputs
+        # cross PCIe into the other set (every step still copies all of its inputs
+        # inside the timed region; only the first copy of the run is exposed)
+        sets = []
+        for a in apps:
+            cur = a["app"].inputs
+            sets.append([cur, [torch.empty_like(t) if t is not None else None for t in cur]])
 
-        def step_e2e():
-            # every app's H2D is issued up front on a copy stream (ps_app_load_host is
-            # asynchronous on its stream), so app k+1's inputs cross PCIe while app k's
-            # sweep runs; each sweep waits only for its own app's copy
+        def issue_copies(k):
+            """H2D of step k's inputs into set k % 2 on the copy stream; one event per app."""
             go = torch.cuda.Event()
-            go.record(stream)
+            go.record(stream)                        # the previous user of that set is done
             copy.wait_event(go)
-            ready = []
-            for a, hin in zip(apps, host):
-                a["app"].load_host(hin, stream=copy)                 # H2D of the inputs
+            evs = []
+            for i, (a, hin) in enumerate(zip(apps, host)):
+                dst = sets[i][k % 2]
+                a["app"].bind(dst, outputs=a["app"].outputs, workspace=a["app"].workspace)
+                a["app"].load_host(hin, stream=copy)                 # H2D into set k % 2
                 ev = torch.cuda.Event()
                 ev.record(copy)
-                ready.append(ev)
-            for a, ev in zip(apps, ready):
+                evs.append(ev)
+            return evs
+
+        def step_e2e(k, ready, last):
+            nxt = None if last else issue_copies(k + 1)
+            for i, (a, ev) in enumerate(zip(apps, ready)):
+                a["app"].bind(sets[i][k % 2], outputs=a["app"].outputs, workspace=a["app"].workspace)
                 stream.wait_event(ev)
                 D.sharded_reference(a["app"], world, rank, refs=a["refs"])
                 arr, _ = a["app"].sweep_raw(a["ids"], args.toq)       # results read back (D2H)
                 if world > 1:
                     D.gather_results(arr)
-        step_e2e()
+            return nxt
+
+        ready = issue_copies(0)                      # warm-up step
+        step_e2e(0, ready, True)
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
         f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         f0.record(stream)
-        for _ in range(args.steps):
-            step_e2e()
+        ready = issue_copies(0)
+        for k in range(args.steps):
+            ready = step_e2e(k, ready, k == args.steps - 1)
         f1.record(stream)
         torch.cuda.synchronize()
         e_ms = f0.elapsed_time(f1)
@@ -740,7 +756,10 @@ def main():
             e_ms = float(t.item())
         e2e = {"value": total_configs * args.steps / (e_ms * 1e-3), "unit": "configs/s",
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "ms_per_step": e_ms / args.steps}
+               "ms_per_step": e_ms / args.steps,
+               "how": "ps_app_load_host of every input (pinned f32) each step on a copy stream into one of "
+                      "two device input sets, overlapped with the previous step's sweep; ps_sweep reads "
+                      "the result records back each app"}
         del host
 
     if rank != 0:

@@ -24,14 +24,8 @@ namespace simt {
 
 namespace {
 constexpr int FBM = 128, FBN = 128, FBK = 16, FST = 3, FTHREADS = 256, FPAD = 4;
-// As rows are 128 + 20 floats: rows 8..15 start 16 floats further in (a_off), so the
-// register-staged k-major A (threads 2i / 2i+1 write rows k / k+8 of column i) hits 32
-// distinct banks (8 * FLA is a multiple of 32 words; without the shift both halves
-// collide: 141M 2-way store conflicts per 8192^3 GEMM in round 1).  The shift is a
-// compile-time constant per unrolled k, so fragment addresses stay immediate offsets.
-constexpr int FLA = FBM + 20, FLB = FBN + FPAD;   // row strides of As[k][m], Bs[k][n]
+constexpr int FLA = FBM + FPAD, FLB = FBN + FPAD;   // row strides of As[k][m], Bs[k][n]
 constexpr int FA_EL = FBK * FLA, FB_EL = FBK * FLB;
-__device__ __forceinline__ int a_off(int k) { return ((k >> 3) & 1) << 4; }
 constexpr int FSMEM = FST * (FA_EL + FB_EL) * 4;
 
 template <class S> __device__ __forceinline__ float widen_f(raw_t<S> v) {
@@ -76,7 +70,7 @@ __global__ void __launch_bounds__(FTHREADS, 2) gemm_ffma_kernel(Params p, float 
       for (int e = 0; e < BM * BK / 4 / THREADS; e++) {
         const int c = tid + e * THREADS;
         const int kr = c / (BM / 4), mc = (c % (BM / 4)) * 4;
-        float *dst = As + kr * LA + mc + a_off(kr);
+        float *dst = As + kr * LA + mc;
         if (fa) {
           cp_async16(dst, Ap + (m0 + mc) * p.a_sr + (k0 + kr) * p.a_sc);
         } else {
@@ -129,8 +123,8 @@ __global__ void __launch_bounds__(FTHREADS, 2) gemm_ffma_kernel(Params p, float 
     if constexpr (!CA) {
 #pragma unroll
       for (int e = 0; e < EA; e++) {
-        if (AK) As[(a_k + e) * LA + a_off(a_k + e) + a_m] = widen_f<SA>(ra[e]);
-        else As[a_k * LA + a_off(a_k) + a_m + e] = widen_f<SA>(ra[e]);
+        if (AK) As[(a_k + e) * LA + a_m] = widen_f<SA>(ra[e]);
+        else As[a_k * LA + a_m + e] = widen_f<SA>(ra[e]);
       }
     }
     if constexpr (!CB) {
@@ -163,8 +157,8 @@ __global__ void __launch_bounds__(FTHREADS, 2) gemm_ffma_kernel(Params p, float 
     const float *As = As0 + st * FA_EL, *Bs = Bs0 + st * FB_EL;
 #pragma unroll
     for (int k = 0; k < BK; k++) {
-      const float4 a0 = *reinterpret_cast<const float4 *>(As + k * LA + a_off(k) + ty * 4);
-      const float4 a1 = *reinterpret_cast<const float4 *>(As + k * LA + a_off(k) + 64 + ty * 4);
+      const float4 a0 = *reinterpret_cast<const float4 *>(As + k * LA + ty * 4);
+      const float4 a1 = *reinterpret_cast<const float4 *>(As + k * LA + 64 + ty * 4);
       const float4 b0 = *reinterpret_cast<const float4 *>(Bs + k * LB + tx * 4);
       const float4 b1 = *reinterpret_cast<const float4 *>(Bs + k * LB + 64 + tx * 4);
       const float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};

@@ -187,3 +187,17 @@ def test_exchange_regions_world3_gloo():
     want[2000:3000] = (np.arange(1000) + 8).astype(np.uint8)
     for _, raw in out:
         assert np.frombuffer(raw, dtype=np.uint8).tobytes() == want.tobytes()
+
+
+@pytest.mark.parametrize("radix", [4, 6])
+def test_partition_bf16_fp8_spaces(radix):
+    """the cost model covers the bf16 (radix 4) and fp8 (radix 6) alphabets --
+    fp8 objects are 1 byte and fp8 x fp8 contractions are costed on tcgen05 f8f6f4."""
+    objs = oracle.app_objects("2mm", [512])
+    ids = list(range(radix ** len(objs)))
+    parts = [D.partition_configs("2mm", [512], objs, ids, 3, r, radix=radix) for r in range(3)]
+    assert sorted(c for p in parts for c in p) == ids
+    if radix == 6:
+        e4 = D.config_cost("2mm", [512], objs, sum(4 * 6 ** m for m in range(5)), 6)
+        f16 = D.config_cost("2mm", [512], objs, sum(2 * 6 ** m for m in range(5)), 6)
+        assert e4 < f16      # fp8 moves half the bytes and runs at twice the tensor rate
