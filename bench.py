@@ -866,6 +866,27 @@ def main():
     else:
         roof, conv_roof = roof_a3, roof_a2
 
+    # modelled multi-GPU scaling (labelled as a model, not a measurement): the partition
+    # dist.partition_configs would use at W ranks (LPT over the cost model), applied to
+    # this run's MEASURED per-configuration device times; the makespan is the slowest
+    # rank's sum.  Excludes the NCCL record gather (64 B per configuration) and setup.
+    scaling_model = None
+    if world == 1:
+        scaling_model = {"how": "LPT partition of the cost model (dist.partition_configs) applied to this "
+                                "run's measured per-configuration total_ms; makespan = slowest rank; "
+                                "model, not a measurement", "speedup": {}}
+        t1 = sum(float(last[a["kind"]]["total_ms"].sum()) for a in apps)
+        for W in (2, 4, 8):
+            ranks = [0.0] * W
+            for a in apps:
+                arr = last[a["kind"]]
+                ms = {int(c): float(t) for c, t in zip(arr["config_id"], arr["total_ms"])}
+                ids = sorted(ms)
+                for r in range(W):
+                    part = D.partition_configs(a["kind"], a["dims"], a["app"].objects, ids, W, r)
+                    ranks[r] += sum(ms[c] for c in part)
+            scaling_model["speedup"][str(W)] = round(t1 / max(ranks), 3)
+
     whole = None
     if not args.no_whole_program and world == 1:
         whole = whole_program(torch, B, apps, args)
@@ -907,6 +928,7 @@ def main():
         "roofline_secondary": conv_roof,
         "conversion_gbs": conv,
         "speedup_vs_fp32_at_toq": speedup,
+        "scaling_model": scaling_model,
         "whole_program": whole,
     }
     print(json.dumps(line), flush=True)
