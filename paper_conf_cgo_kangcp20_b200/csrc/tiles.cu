@@ -44,8 +44,19 @@ struct TileArgs {
   int vec_ok;
 };
 
+// Minimum CTAs per SM for __launch_bounds__: 16-bit A with f32 arithmetic and row
+// dots (8-row groups) is capped at 80 registers so THREE CTAs share an SM -- these
+// statements are bound by global-load latency (ncu: long_scoreboard 57% of stalls,
+// 14 of 64 warps active), so 50% more warps in flight is what they need.  0 = not
+// specified (ptxas keeps its default, <= 128 registers here; an explicit 1 lets it
+// grow to ~230 and halves the occupancy of the f64 statements)
+template <class SA, class TC, class TR, bool RD>
+constexpr int tile_minb() {
+  return (RD && sizeof(raw_t<SA>) == 2 && sizeof(TC) == 4 && sizeof(TR) == 4) ? 3 : 0;
+}
+
 template <class SA, class TC, class TR, int CM, bool RD>
-__global__ void __launch_bounds__(TTHREADS) tile_kernel(TileArgs a) {
+__global__ void __launch_bounds__(TTHREADS, tile_minb<SA, TC, TR, RD>()) tile_kernel(TileArgs a) {
   using RA = raw_t<SA>;
   constexpr int V = 16 / sizeof(RA);
   constexpr bool SAME = std::is_same<TC, TR>::value;
