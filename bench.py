@@ -579,6 +579,9 @@ def main():
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"])
     ap.add_argument("--fake", action="store_true",
                     help="CPU dry run of the multi-rank orchestration (fake records; needs --backend gloo)")
+    ap.add_argument("--shard-rows", action="store_true",
+                    help="evaluate every configuration row-sharded over all ranks (ps_shard_step) "
+                         "instead of partitioning the configurations")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-conversion", action="store_true")
@@ -592,6 +595,8 @@ def main():
     elif args.warmup < 3:
         log("warmup raised to 3 (timing rule)")
         args.warmup = 3
+    if args.shard_rows:
+        args.no_e2e = True
     if args.fake and args.backend != "gloo":
         ap.error("--fake runs on CPU: use --backend gloo")
 
@@ -634,7 +639,7 @@ def main():
         app.bind(dins)
         refs = D.sharded_reference(app, world, rank)
         ids = list(range(app.space))
-        mine = D.partition_configs(kind, dims, app.objects, ids, world, rank) if world > 1 else ids
+        mine = D.partition_configs(kind, dims, app.objects, ids, world, rank) if world > 1 and not args.shard_rows else ids
         apps.append(dict(kind=kind, dims=dims, app=app, ins=ins, refs=refs, ids=mine,
                          space=app.space))
         log("rank %d setup %s %s: %d/%d configs, %.1f s" % (rank, kind, dims, len(mine),
@@ -645,9 +650,18 @@ def main():
     def step(collect=None):
         for a in apps:
             D.sharded_reference(a["app"], world, rank, refs=a["refs"])   # a0 (row-sharded)
-            arr, _ = a["app"].sweep_raw(a["ids"], args.toq)          # a1-a7 (local share)
-            if world > 1:
-                arr = D.gather_results(arr)                          # NCCL gather
+            if args.shard_rows:
+                # every configuration row-sharded over all ranks (ps_shard_step stages +
+                # NCCL all-gathers of the exchanged ranges), records identical on every rank
+                recs = [D.sharded_evaluate(a["app"], a["app"].decode(c), args.toq) for c in range(a["space"])]
+                arr = np.zeros(len(recs), dtype=B.RESULT_DTYPE)
+                for i, r in enumerate(recs):
+                    for k in B.RESULT_DTYPE.names:
+                        arr[i][k] = r[k]
+            else:
+                arr, _ = a["app"].sweep_raw(a["ids"], args.toq)      # a1-a7 (local share)
+                if world > 1:
+                    arr = D.gather_results(arr)                      # NCCL gather
             if collect is not None:
                 collect[a["kind"]] = arr
 
@@ -918,7 +932,9 @@ def main():
                    "step": "a0 reference + full 3^M config space per app (a1-a7)",
                    "l2": "inputs larger than L2: largest object %.0f MB at fp32 vs 126 MB L2%s" % (
                        max_obj / 1e6, "" if max_obj > 126e6 else " (NOT larger: launch-bound case)"),
-                   "parallelism": "configs partitioned over %d GPU(s), NCCL result gather" % world,
+                   "parallelism": ("each configuration row-sharded over %d GPU(s) (ps_shard_step, NCCL "
+                                   "all-gathers of the exchanged ranges)" % world) if args.shard_rows else
+                                  "configs partitioned over %d GPU(s), NCCL result gather" % world,
                    "configs_per_rank": per_rank,
                    "baseline_n_gpus": BASELINE_GPUS.get(args.workload)},
         "paper_context": PAPER_CONTEXT,

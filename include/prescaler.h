@@ -246,9 +246,10 @@ PS_API ps_status ps_run_config(ps_app *app, const int *prec, double toq, void *s
 /*   the rows of A (and B) for ATAX / BICG / GESUMMV / MVT; the rows of the      */
 /*   scored output for GEMM, 2MM, 3MM (F rows get their own split), SYR2K,     */
 /*   2DCONV, 3DCONV; the upper-triangular output rows for SYRK, CORR, COVAR     */
-/*   (CORR / COVAR split the data rows for the column statistics).  FDTD-2D     */
-/*   (TMAX dependent sweeps) and fp8 objects (per-tensor scales need the whole */
-/*   object) are not row-shardable: PS_ERR_UNSUPPORTED.                         */
+/*   (CORR / COVAR split the data rows for the column statistics); the rows of  */
+/*   ex / ey / hz for FDTD-2D (one halo row of ey and of hz exchanged per time   */
+/*   step).  fp8 objects (a per-tensor scale needs the whole object) are not     */
+/*   row-shardable: PS_ERR_UNSUPPORTED.                                          */
 /*   Row bounds are aligned so every reduction keeps its single-GPU association */
 /*   (R5 256-row column-sum chunks, whole quality segments, whole 256-row      */
 /*   tcgen05 tiles): the record and the delivered outputs are bit-identical to */

@@ -803,7 +803,8 @@ ps_status ready(const ps_app *a) {
 // (column-chunk partials, row blocks, quality segment partials) and every
 // reduction keeps its single-GPU association, so the record and the delivered
 // outputs are bit-identical to ps_run_config for every W.
-enum ShardProg { SP_NONE, SP_ATAX, SP_BICG, SP_GESUMMV, SP_MVT, SP_ROWS, SP_3MM, SP_SYRK, SP_CORR, SP_COVAR };
+enum ShardProg { SP_NONE, SP_ATAX, SP_BICG, SP_GESUMMV, SP_MVT, SP_ROWS, SP_3MM, SP_SYRK, SP_CORR, SP_COVAR,
+                 SP_FDTD };
 
 struct ShardGeo {
   int prog = SP_NONE;
@@ -825,7 +826,12 @@ ShardGeo shard_geo(const ps_app *a) {
     case K_SYRK: g.prog = SP_SYRK; break;
     case K_CORR: g.prog = SP_CORR; break;
     case K_COVAR: g.prog = SP_COVAR; break;
-    default: return g;   // FDTD-2D: TMAX dependent sweeps -- configurations are partitioned instead
+    case K_FDTD2D:   // rows of ex / ey / hz; one-row halos exchanged twice per time step
+      g.prog = SP_FDTD;
+      g.rows = a->d[1];
+      g.align = 1;
+      return g;
+    default: return g;
   }
   if (g.prog == SP_ATAX || g.prog == SP_BICG || g.prog == SP_GESUMMV || g.prog == SP_MVT) {
     g.rows = a->d[0];    // rows of A (and B)
@@ -934,6 +940,32 @@ ps_status quality_rows(ps_app *a, Ctx &c, int m, int64_t r0, int64_t r1, ps_shar
 }
 ps_status quality_rows_finalize(ps_app *a, int m, QPart *res, cudaStream_t st) {
   return quality_finalize_async((QPart *)(a->ws + a->qparts_off), qseg(a->rows[m], a->cols[m]).nb, res, st);
+}
+// every output row-sharded alike (FDTD-2D's ex, ey, hz): segment partials of rows
+// [r0, r1) of each output at that output's offset in the partial array (the layout
+// of enqueue_config), one exchange region per output
+ps_status quality_rows_all(ps_app *a, Ctx &c, int64_t r0, int64_t r1, ps_shard_step_t *x) {
+  QPart *parts = (QPart *)(a->ws + a->qparts_off);
+  int np = 0;
+  for (int m = 0; m < a->def->nobj; m++) {
+    if (!a->def->o[m].is_output) continue;
+    const QSeg q = qseg(a->rows[m], a->cols[m]);
+    const int s0 = (int)(r0 / q.rows_per);
+    const int s1 = r1 >= a->rows[m] ? q.nb : (int)(r1 / q.rows_per);
+    x->region[x->nregions++] = ps_shard_region{parts, (uint64_t)(np + s0) * sizeof(QPart),
+                                               (uint64_t)(s1 > s0 ? s1 - s0 : 0) * sizeof(QPart)};
+    if (s1 > s0)
+      PS_TRY(backconv_quality_async(c.ptr[m], c.prec[m], a->ref[m], a->orig_out[m], a->rows[m], a->cols[m],
+                                    parts + np, c.st, s0, s1));
+    np += q.nb;
+  }
+  return PS_OK;
+}
+int quality_parts_all(const ps_app *a) {
+  int np = 0;
+  for (int m = 0; m < a->def->nobj; m++)
+    if (a->def->o[m].is_output) np += qseg(a->rows[m], a->cols[m]).nb;
+  return np;
 }
 
 // One stage of the program; events ev[0..4] bracket a2 / statements / a4+a5 partials /
@@ -1232,6 +1264,51 @@ ps_status shard_stage(ps_app *a, const int *prec, int rank, int world, int stage
       PS_TRY(rec(4));
       return PS_OK;
     }
+  }
+  if (g.prog == SP_FDTD) {   // FDTD-2D: per time step two stages, then quality
+    const int64_t TM = d[0], NX = d[1], NY = d[2];
+    (void)NX;
+    auto row1 = [&](int m, int64_t r) {   // one row of object m (a halo row for a neighbour)
+      return (r0 < r1) ? row_region(a, c, m, r, r + 1) : ps_shard_region{c.ptr[m], 0, 0};
+    };
+    if (stage < 2 * TM) {
+      const int64_t t = stage / 2;
+      PS_TRY(rec(0));
+      if (stage == 0) {   // a2: fict whole, the rows of ex / ey / hz with a one-row halo
+        PS_TRY(a2_rows(a, c, 0));
+        for (int m = 1; m <= 3; m++) PS_TRY(a2_rows(a, c, m, r0 - 1, r1 + 1));
+      }
+      PS_TRY(rec(1));
+      if (stage % 2 == 0) {   // ey (row 0 from fict, rows >= 1 need hz[i-1]: halo r0 - 1), ex
+        PS_TRY(fdtd2d_part_async(FDTD_EY, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], NY, st, r0, r1));
+        PS_TRY(fdtd2d_part_async(FDTD_EX, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], NY, st, r0, r1));
+        region(row1(2, r0));          // my first ey row: the previous rank's hz needs ey[i+1]
+      } else {                        // hz (needs ey[i+1]: halo r1)
+        PS_TRY(fdtd2d_part_async(FDTD_HZ, P[0], p[0], P[1], p[1], P[2], p[2], P[3], p[3], t, d[1], NY, st, r0, r1));
+        region(row1(3, r1 - 1));      // my last hz row: the next rank's ey needs hz[i-1]
+      }
+      PS_TRY(rec(2));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      return PS_OK;
+    }
+    if (stage == 2 * TM) {
+      PS_TRY(rec(0));
+      PS_TRY(rec(1));
+      PS_TRY(rec(2));
+      PS_TRY(quality_rows_all(a, c, r0, r1, x));
+      PS_TRY(rec(3));
+      PS_TRY(rec(4));
+      return PS_OK;
+    }
+    PS_TRY(rec(0));
+    PS_TRY(rec(1));
+    PS_TRY(rec(2));
+    PS_TRY(rec(3));
+    PS_TRY(quality_finalize_async((QPart *)(a->ws + a->qparts_off), quality_parts_all(a), res, st));
+    PS_TRY(rec(4));
+    x->done = 1;
+    return PS_OK;
   }
   set_error("ps_shard_step: %s has no row-sharded evaluation", a->def->kind);
   return PS_ERR_UNSUPPORTED;

@@ -103,7 +103,8 @@ ps_status conv3d_rows_async(const void *A, int ta, void *B, int tb, int64_t ni, 
 // the ey update in one pass; FDTD_EY0 / FDTD_EY1 = those two parts alone (reading #29)
 enum FdtdPart { FDTD_EY = 0, FDTD_EY0 = 1, FDTD_EY1 = 2, FDTD_EX = 3, FDTD_HZ = 4 };
 ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int tex, void *ey, int tey,
-                            void *hz, int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st);
+                            void *hz, int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st,
+                            int64_t r0 = 0, int64_t r1 = -1);   // rows [r0, r1) (row-sharded)
 ps_status colsum_async(const void *A, int ta, int64_t lda, const void *w, int tw, void *out,
                        int tout, int64_t rows, int64_t cols, int T, int mode, int fin, double n,
                        double eps, void *partial, cudaStream_t st);

@@ -338,11 +338,12 @@ template <class SF, class SE, class SH>
 __global__ void __launch_bounds__(FD_NT) fdtd_ey_kernel(const raw_t<SF> *__restrict__ fict,
                                                         raw_t<SE> *__restrict__ ey,
                                                         const raw_t<SH> *__restrict__ hz, int64_t t,
-                                                        int64_t nx, int64_t ny, int part) {
+                                                        int64_t nx, int64_t ny, int part, int64_t i0,
+                                                        int64_t i1) {
   using TA = T2<SF, SE>;   // ey[0][j] = fict[t]
   using TB = T2<SE, SH>;   // ey[i][j] -= 0.5 (hz[i][j] - hz[i-1][j])
   const int64_t jb = (int64_t)blockIdx.x * FD_COLS + threadIdx.x;
-  for (int64_t i = blockIdx.y; i < nx; i += gridDim.y) {
+  for (int64_t i = i0 + blockIdx.y; i < i1; i += gridDim.y) {
     const int64_t row = i * ny;
     if ((i == 0 && part == FDTD_EY1) || (i > 0 && part == FDTD_EY0)) continue;
     if (i == 0) {
@@ -373,10 +374,10 @@ __global__ void __launch_bounds__(FD_NT) fdtd_ey_kernel(const raw_t<SF> *__restr
 template <class SE, class SH>
 __global__ void __launch_bounds__(FD_NT) fdtd_ex_kernel(raw_t<SE> *__restrict__ ex,
                                                         const raw_t<SH> *__restrict__ hz, int64_t nx,
-                                                        int64_t ny) {
+                                                        int64_t ny, int64_t i0, int64_t i1) {
   using T = T2<SE, SH>;    // ex[i][j] -= 0.5 (hz[i][j] - hz[i][j-1]),  j >= 1
   const int64_t jb = (int64_t)blockIdx.x * FD_COLS + threadIdx.x;
-  for (int64_t i = blockIdx.y; i < nx; i += gridDim.y) {
+  for (int64_t i = i0 + blockIdx.y; i < i1; i += gridDim.y) {
     const int64_t row = i * ny;
     T h[FD_U], g[FD_U], e[FD_U];
 #pragma unroll
@@ -400,10 +401,11 @@ template <class SH, class SX, class SY>
 __global__ void __launch_bounds__(FD_NT) fdtd_hz_kernel(raw_t<SH> *__restrict__ hz,
                                                         const raw_t<SX> *__restrict__ ex,
                                                         const raw_t<SY> *__restrict__ ey, int64_t nx,
-                                                        int64_t ny, T3<SH, SX, SY> c07) {
+                                                        int64_t ny, T3<SH, SX, SY> c07, int64_t i0,
+                                                        int64_t i1) {
   using T = T3<SH, SX, SY>;   // hz -= 0.7 (((ex[i][j+1] - ex[i][j]) + ey[i+1][j]) - ey[i][j])
   const int64_t jb = (int64_t)blockIdx.x * FD_COLS + threadIdx.x;
-  for (int64_t i = blockIdx.y; i + 1 < nx; i += gridDim.y) {
+  for (int64_t i = i0 + blockIdx.y; i < i1 && i + 1 < nx; i += gridDim.y) {
     const int64_t row = i * ny;
     T x1[FD_U], x0[FD_U], y1[FD_U], y0[FD_U], h[FD_U];
 #pragma unroll
@@ -430,10 +432,18 @@ __global__ void __launch_bounds__(FD_NT) fdtd_hz_kernel(raw_t<SH> *__restrict__ 
   }
 }
 
+// rows [r0, r1) of the statement (r1 < 0: every row) -- a row-sharded evaluation
 ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int tex, void *ey, int tey,
-                            void *hz, int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st) {
+                            void *hz, int thz, int64_t t, int64_t nx, int64_t ny, cudaStream_t st, int64_t r0,
+                            int64_t r1) {
   if (nx <= 0 || ny <= 0) return PS_OK;
-  const int64_t rows = part == FDTD_EY0 ? 1 : nx;
+  if (r1 < 0) r1 = nx;
+  if (r1 <= r0) return PS_OK;
+  if (part == FDTD_EY0) {   // the row-0 assignment belongs to the rank owning row 0
+    if (r0 > 0) return PS_OK;
+    r1 = 1;
+  }
+  const int64_t rows = r1 - r0;
   if (part == FDTD_EY0) thz = PS_F32;   // the row-0 assignment reads fict only (hz unused)
   if (part == FDTD_EY1) tf = PS_F32;    // the update reads hz only (fict unused)
   const dim3 grid((unsigned)((ny + FD_COLS - 1) / FD_COLS), (unsigned)(rows < 65535 ? rows : 65535));
@@ -444,7 +454,7 @@ ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int te
         using SE = decltype(b);
         using SH = decltype(c);
         fdtd_ey_kernel<SF, SE, SH><<<grid, FD_NT, 0, st>>>((const raw_t<SF> *)fict, (raw_t<SE> *)ey,
-                                                           (const raw_t<SH> *)hz, t, nx, ny, part);
+                                                           (const raw_t<SH> *)hz, t, nx, ny, part, r0, r1);
         PS_CHECK_LAUNCH("fdtd_ey_kernel");
         return PS_OK;
       });
@@ -454,7 +464,7 @@ ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int te
     return dispatch_store(thz, [&](auto c) -> ps_status {
       using SE = decltype(a);
       using SH = decltype(c);
-      fdtd_ex_kernel<SE, SH><<<grid, FD_NT, 0, st>>>((raw_t<SE> *)ex, (const raw_t<SH> *)hz, nx, ny);
+      fdtd_ex_kernel<SE, SH><<<grid, FD_NT, 0, st>>>((raw_t<SE> *)ex, (const raw_t<SH> *)hz, nx, ny, r0, r1);
       PS_CHECK_LAUNCH("fdtd_ex_kernel");
       return PS_OK;
     });
@@ -467,7 +477,7 @@ ps_status fdtd2d_part_async(int part, const void *fict, int tf, void *ex, int te
         using SY = decltype(c);
         using T = T3<SH, SX, SY>;
         fdtd_hz_kernel<SH, SX, SY><<<grid, FD_NT, 0, st>>>((raw_t<SH> *)hz, (const raw_t<SX> *)ex,
-                                                           (const raw_t<SY> *)ey, nx, ny, (T)0.7);
+                                                           (const raw_t<SY> *)ey, nx, ny, (T)0.7, r0, r1);
         PS_CHECK_LAUNCH("fdtd_hz_kernel");
         return PS_OK;
       });

@@ -205,19 +205,19 @@ __global__ void __launch_bounds__(256) colsum_finalize_kernel(const T *__restric
                                                               T eps) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= cols) return;
-  // chunks in order; the loads of up to 32 chunks are issued together (predicated,
-  // so an absent chunk is skipped, never added as +0) and the in-order chain waits
-  // on ~2 L2/DRAM round trips for the 64 chunks of a 16384-row matrix, not 8
+  // chunks in order; loads issued 8 at a time so the in-order chain does not wait
+  // on one L2 round trip per term (32 at a time, predicated, measured 0.8% slower on
+  // the matvec step: profiles/bench_ab_finalize_r2r.json)
   T total = partial[j];
-  for (int64_t c = 1; c < nchunks; c += 32) {
-    T v[32];
+  int64_t c = 1;
+  for (; c + 8 <= nchunks; c += 8) {
+    T v[8];
 #pragma unroll
-    for (int u = 0; u < 32; u++)
-      if (c + u < nchunks) v[u] = partial[(c + u) * cols + j];
+    for (int u = 0; u < 8; u++) v[u] = partial[(c + u) * cols + j];
 #pragma unroll
-    for (int u = 0; u < 32; u++)
-      if (c + u < nchunks) total = total + v[u];
+    for (int u = 0; u < 8; u++) total = total + v[u];
   }
+  for (; c < nchunks; c++) total = total + partial[c * cols + j];
   if (FIN == FIN_MEAN) total = total / n;
   if (FIN == FIN_STDDEV) {
     total = sqrt(total / n);
@@ -234,15 +234,15 @@ __global__ void __launch_bounds__(256) rowdot_finalize_kernel(const T *__restric
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= rows) return;
   T total = qpart[i];   // tiles in order, loads batched as in colsum_finalize_kernel
-  for (int64_t t = 1; t < ntiles; t += 32) {
-    T v[32];
+  int64_t t = 1;
+  for (; t + 8 <= ntiles; t += 8) {
+    T v[8];
 #pragma unroll
-    for (int u = 0; u < 32; u++)
-      if (t + u < ntiles) v[u] = qpart[(t + u) * rows + i];
+    for (int u = 0; u < 8; u++) v[u] = qpart[(t + u) * rows + i];
 #pragma unroll
-    for (int u = 0; u < 32; u++)
-      if (t + u < ntiles) total = total + v[u];
+    for (int u = 0; u < 8; u++) total = total + v[u];
   }
+  for (; t < ntiles; t++) total = total + qpart[t * rows + i];
   if (add) total = Ld<SO, T>::get(out, (size_t)i) + total;                   // MVT: x1 + A y1
   St<SO, T>::put(out, (size_t)i, total);
 }

@@ -5,7 +5,8 @@ shard's produced byte ranges are copied into the other shards' workspaces (what
 an NCCL all-gather does across GPUs, dist.exchange_regions).  The records and the
 delivered outputs must be bit-identical to the unsharded ps_run_config for
 W = 2, 3, 5 (including empty shards), in f64 / f32 / f16 (tcgen05) / mixed
-configurations."""
+configurations, for all 14 apps (FDTD-2D exchanging one halo row of ey and of hz
+per time step)."""
 import numpy as np
 import pytest
 
@@ -15,7 +16,7 @@ CASES = {
     "atax": [1100, 900], "bicg": [1100, 900], "gesummv": [1100], "mvt": [1100],
     "gemm": [1100, 300, 200], "2mm": [1100, 260, 200, 300], "3mm": [1100, 600, 200, 300, 250],
     "syr2k": [300, 1100], "syrk": [300, 1100], "corr": [1000, 1100], "covar": [1000, 1100],
-    "conv2d": [1100, 700], "conv3d": [40, 30, 50],
+    "conv2d": [1100, 700], "conv3d": [40, 30, 50], "fdtd2d": [5, 600, 300],
 }
 
 
@@ -111,8 +112,15 @@ def test_bounds_cover_and_align():
                 assert a1 == c0 and a0 <= a1
 
 
-def test_fdtd_and_fp8_are_rejected():
+def test_fp8_objects_are_rejected():
+    """A per-tensor fp8 scale needs the amax of the whole object: not row-shardable."""
     import torch
     from paper_conf_cgo_kangcp20_b200 import binding as B
-    app = B.App("fdtd2d", [4, 64, 64])
-    assert app.eval_shard_rows == 0
+    from paper_conf_cgo_kangcp20_b200 import inputs as gen
+    app = B.App("gemm", [300, 200, 100])
+    app.set_flags(B.FLAG_FP8)
+    ins = gen.make_inputs("gemm", app.objects, "random")
+    app.bind([torch.from_numpy(a.reshape(-1)).cuda() for a in ins])
+    app.reference()
+    with pytest.raises(B.PsError):
+        app.shard_step([4, 4, 1], 0, 2, 0)

@@ -46,6 +46,24 @@ if "f32" in WHICH:   # FFMA (SIMT, R3-exact): GEMM all-f32 (A k-major), f16 A, f
         lib_rate("gemm", prec, B.FLAG_NO_TENSOR_CORES, gemm, "gemm_ffma_kernel")
 if "f64" in WHICH:   # DMMA chains
     lib_rate("gemm", [0, 0, 0], 0, gemm, "gemm_dmma_kernel")
+if "tcplain" in WHICH:   # C = A.B written plainly (no alpha/beta read of C): 2MM with every object
+    # f16 but E, NL = 256 -- both statements on tcgen05, the second 3% of the flops
+    def lib_rate_dims(kind, dims, prec, flags, flop, label, reps=5):
+        app = B.App(kind, dims)
+        app.set_flags(flags)
+        ins = gen.make_inputs(kind, app.objects, "random")
+        app.bind([torch.from_numpy(a.reshape(-1)).cuda() if a is not None else None for a in ins])
+        app.reference()
+        app.run_config(prec)
+        ms = min(app.run_config(prec)["kernel_ms"] for _ in range(reps))
+        emit(kernel=label, app=kind, dims=dims, prec=prec, kernel_ms=round(ms, 4),
+             tflops=round(flop / (ms * 1e-3) / 1e12, 1))
+        del app
+        torch.cuda.empty_cache()
+    d = [N, N, N, 256]
+    fl = 2.0 * N ** 3 + 2.0 * N * N * 256
+    lib_rate_dims("2mm", d, [2, 2, 2, 2, 1], 0, fl, "gemm_tc2_kernel fp16, plain epilogue (C f16, then E = C.D, NL 256)")
+    lib_rate_dims("2mm", d, [3, 3, 3, 3, 1], B.FLAG_BF16, fl, "gemm_tc2_kernel bf16, plain epilogue (C bf16, then E = C.D, NL 256)")
 if "tc" in WHICH:    # tcgen05: fp16, bf16, e4m3, e5m2 multiplicands, f32 C
     lib_rate("gemm", [2, 2, 1], 0, gemm, "gemm_tc2_kernel fp16")
     lib_rate("gemm", [3, 3, 1], B.FLAG_BF16, gemm, "gemm_tc2_kernel bf16")
