@@ -355,6 +355,8 @@ typedef struct {
   int32_t trials;         /* distinct configurations executed (RunApp calls)    */
   uint64_t pfp_id;        /* PFP starting configuration                         */
   uint64_t trial_ids[64]; /* executed configurations in order (first 64)        */
+  float trial_ms[64];     /* their median measured times (RunApp's time)        */
+  int32_t trial_pass[64]; /* their TOQ decisions (Alg. 1 line 10)               */
 } ps_search_result;
 PS_API ps_status ps_search(ps_app *app, double toq, int repeats, void *stream,
                            ps_search_result *out);

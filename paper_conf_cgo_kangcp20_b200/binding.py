@@ -79,7 +79,8 @@ class PsSearchResult(ctypes.Structure):
     _fields_ = [("config_id", ctypes.c_uint64), ("total_ms", ctypes.c_float),
                 ("pfp_ms", ctypes.c_float), ("quality", ctypes.c_double), ("pass_", ctypes.c_int32),
                 ("trials", ctypes.c_int32), ("pfp_id", ctypes.c_uint64),
-                ("trial_ids", ctypes.c_uint64 * 64)]
+                ("trial_ids", ctypes.c_uint64 * 64), ("trial_ms", ctypes.c_float * 64),
+                ("trial_pass", ctypes.c_int32 * 64)]
 
 
 RESULT_DTYPE = np.dtype([("config_id", "<u8"), ("convert_ms", "<f4"), ("kernel_ms", "<f4"),
@@ -452,7 +453,9 @@ class App:
         return {"config_id": int(r.config_id), "prec": self.decode(r.config_id),
                 "total_ms": float(r.total_ms), "quality": float(r.quality), "pass": bool(r.pass_),
                 "trials": int(r.trials), "pfp_id": int(r.pfp_id), "pfp_ms": float(r.pfp_ms),
-                "trial_ids": [int(x) for x in r.trial_ids[:min(r.trials, 64)]]}
+                "trial_ids": [int(x) for x in r.trial_ids[:min(r.trials, 64)]],
+                "trial_ms": [float(x) for x in r.trial_ms[:min(r.trials, 64)]],
+                "trial_pass": [bool(x) for x in r.trial_pass[:min(r.trials, 64)]]}
 
     def sweep(self, config_ids, toq: float = 0.9, stream=None):
         arr, best = self.sweep_raw(config_ids, toq, stream)

@@ -1742,7 +1742,11 @@ ps_status ps_search(ps_app *a, double toq, int repeats, void *stream, ps_search_
     std::sort(ms.begin(), ms.end());
     *t = Trial{ms[ms.size() / 2], r.quality, r.pass != 0};
     seen[id] = *t;
-    if (out->trials < 64) out->trial_ids[out->trials] = id;
+    if (out->trials < 64) {
+      out->trial_ids[out->trials] = id;
+      out->trial_ms[out->trials] = t->ms;
+      out->trial_pass[out->trials] = t->pass;
+    }
     out->trials++;
     return PS_OK;
   };

@@ -88,6 +88,14 @@ if "cublas" in WHICH:
         ms = tm(lambda: a @ b)
         emit(kernel="cuBLAS matmul", dtype=str(dt), N=N, kernel_ms=round(ms, 4), tflops=round(gemm / (ms * 1e-3) / 1e12, 1))
         del a, b
+    # f32 with TF32 off: cuBLAS's own FFMA SGEMM, the practical ceiling for gemm_ffma_kernel
+    torch.backends.cuda.matmul.allow_tf32 = False
+    a = torch.randn(N, N, device="cuda")
+    b = torch.randn(N, N, device="cuda")
+    ms = tm(lambda: a @ b, reps=3)
+    emit(kernel="cuBLAS matmul (FFMA, tf32 off)", dtype="torch.float32", N=N, kernel_ms=round(ms, 4),
+         tflops=round(gemm / (ms * 1e-3) / 1e12, 1))
+    del a, b
     try:
         a = torch.randn(N, N, device="cuda").to(torch.float8_e4m3fn)
         b = torch.randn(N, N, device="cuda").to(torch.float8_e4m3fn).t()
