@@ -38,7 +38,7 @@ __global__ void ref_kernel(const float *A, const float *B, float *C, int M, int 
   C[(size_t)m * N + n] = acc;
 }
 
-template <int BM, int BN, int BK, int TM, int TN, int THREADS, int S, int MINB, bool DB>
+template <int BM, int BN, int BK, int TM, int TN, int THREADS, int S, int MINB, bool DB, bool F2 = false>
 __global__ void __launch_bounds__(THREADS, MINB) ffma_kernel(const float *__restrict__ A, const float *__restrict__ B,
                                                              float *__restrict__ C, int M, int N, int K) {
   constexpr int TX = BN / TN, TY = BM / TM;
@@ -46,7 +46,6 @@ __global__ void __launch_bounds__(THREADS, MINB) ffma_kernel(const float *__rest
   constexpr int LA = BM + 4, LB = BN + 4;
   constexpr int AEL = BK * LA, BEL = BK * LB;
   constexpr int EA = BM * BK / THREADS;            // A elements per thread per tile
-  constexpr int RUNS = BK / EA;                    // threads per A row
   static_assert(EA % 4 == 0 && BK % EA == 0, "A run");
   extern __shared__ __align__(16) float sm[];
   float *As0 = sm, *Bs0 = sm + S * AEL;
@@ -80,11 +79,17 @@ __global__ void __launch_bounds__(THREADS, MINB) ffma_kernel(const float *__rest
       cp16(Bs + kr * LB + nc, B + (size_t)(kt * BK + kr) * N + n0 + nc);
     }
   };
-  float acc[TM][TN];
+  float2 acc[TM][TN / 2];
 #pragma unroll
   for (int i = 0; i < TM; i++)
 #pragma unroll
-    for (int j = 0; j < TN; j++) acc[i][j] = 0.f;
+    for (int j = 0; j < TN / 2; j++) acc[i][j] = make_float2(0.f, 0.f);
+  // one output pair (columns 2j, 2j+1): FFMA2 (fma.rn.f32x2 = two independent fma.rn,
+  // bit-identical to two FFMAs) with a[i] broadcast, or two FFMAs
+  auto fma_pair = [&](float a, float b0, float b1, float2 &c) {
+    if constexpr (F2) c = __ffma2_rn(make_float2(a, a), make_float2(b0, b1), c);
+    else { c.x = __fmaf_rn(a, b0, c.x); c.y = __fmaf_rn(a, b1, c.y); }
+  };
 
 #pragma unroll
   for (int s = 0; s < S - 1; s++) {
@@ -119,7 +124,7 @@ __global__ void __launch_bounds__(THREADS, MINB) ffma_kernel(const float *__rest
 #pragma unroll
         for (int i = 0; i < TM; i++)
 #pragma unroll
-          for (int j = 0; j < TN; j++) acc[i][j] = __fmaf_rn(a[k & 1][i], b[k & 1][j], acc[i][j]);
+          for (int j = 0; j < TN / 2; j++) fma_pair(a[k & 1][i], b[k & 1][2 * j], b[k & 1][2 * j + 1], acc[i][j]);
       }
     } else {
 #pragma unroll
@@ -138,7 +143,7 @@ __global__ void __launch_bounds__(THREADS, MINB) ffma_kernel(const float *__rest
 #pragma unroll
         for (int i = 0; i < TM; i++)
 #pragma unroll
-          for (int j = 0; j < TN; j++) acc[i][j] = __fmaf_rn(a[i], b[j], acc[i][j]);
+          for (int j = 0; j < TN / 2; j++) fma_pair(a[i], b[2 * j], b[2 * j + 1], acc[i][j]);
       }
     }
     if (nt < ktiles) store_a(nt % S);
@@ -151,16 +156,16 @@ __global__ void __launch_bounds__(THREADS, MINB) ffma_kernel(const float *__rest
     for (int j4 = 0; j4 < TN / 4; j4++) {
       const int gn = n0 + j4 * TX * 4 + tx * 4;
       *reinterpret_cast<float4 *>(C + (size_t)gm * N + gn) =
-          make_float4(acc[i][j4 * 4], acc[i][j4 * 4 + 1], acc[i][j4 * 4 + 2], acc[i][j4 * 4 + 3]);
+          make_float4(acc[i][j4 * 2].x, acc[i][j4 * 2].y, acc[i][j4 * 2 + 1].x, acc[i][j4 * 2 + 1].y);
     }
   }
 }
 
 static float *dA, *dB, *dC, *dR;
 
-template <int BM, int BN, int BK, int TM, int TN, int THREADS, int S, int MINB, bool DB>
+template <int BM, int BN, int BK, int TM, int TN, int THREADS, int S, int MINB, bool DB, bool F2 = false>
 void run(const char *name, int n) {
-  auto k = ffma_kernel<BM, BN, BK, TM, TN, THREADS, S, MINB, DB>;
+  auto k = ffma_kernel<BM, BN, BK, TM, TN, THREADS, S, MINB, DB, F2>;
   const int smem = S * BK * ((BM + 4) + (BN + 4)) * 4;
   CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   cudaFuncAttributes fa;
@@ -226,5 +231,30 @@ int main(int argc, char **argv) {
   V("H 128x128 t128 16x8 bk8 s6 minb2", 128, 128, 8, 16, 8, 128, 6, 2, false);
   V("I 128x256 t256 8x16 bk16 s3 minb1", 128, 256, 16, 8, 16, 256, 3, 1, false);
   V("J 128x64 t128 8x8 bk16 s4 minb4", 128, 64, 16, 8, 8, 128, 4, 4, false);
+  V("P A+ffma2 128x128 t256 8x8 bk16 s3 minb2", 128, 128, 16, 8, 8, 256, 3, 2, false, true);
+  V("Q C+ffma2 128x128 t128 16x8 bk16 s4 minb2", 128, 128, 16, 16, 8, 128, 4, 2, false, true);
+  V("R F+ffma2 256x128 t256 16x8 bk16 s4 minb1", 256, 128, 16, 16, 8, 256, 4, 1, false, true);
+  V("S E+ffma2 128x128 t128 8x16 bk16 s4 minb2", 128, 128, 16, 8, 16, 128, 4, 2, false, true);
+  V("T I+ffma2 128x256 t256 8x16 bk16 s3 minb1", 128, 256, 16, 8, 16, 256, 3, 1, false, true);
+  V("U 128x64 t128 8x8 bk16 s4 minb3 ffma2", 128, 64, 16, 8, 8, 128, 4, 3, false, true);
+  V("W 128x128 t256 8x8 bk8 s4 minb2 ffma2", 128, 128, 8, 8, 8, 256, 4, 2, false, true);
+  V("X 128x128 t128 16x8 bk8 s6 minb2 ffma2", 128, 128, 8, 16, 8, 128, 6, 2, false, true);
+  V("Y 128x128 t256 8x8 bk16 s3 minb2 db ffma2", 128, 128, 16, 8, 8, 256, 3, 2, true, true);
+  V("Z1 128x64 t128 8x8 bk16 s3 minb2 ffma2", 128, 64, 16, 8, 8, 128, 3, 2, false, true);
+  V("Z2 128x64 t128 8x8 bk16 s3 minb2 db ffma2", 128, 64, 16, 8, 8, 128, 3, 2, true, true);
+  V("Z3 128x64 t128 8x8 bk8 s4 minb2 db ffma2", 128, 64, 8, 8, 8, 128, 4, 2, true, true);
+  V("Z4 128x128 t128 16x8 bk8 s6 minb2 db ffma2", 128, 128, 8, 16, 8, 128, 6, 2, true, true);
+  V("Z5 128x256 t256 8x16 bk16 s3 minb1 db ffma2", 128, 256, 16, 8, 16, 256, 3, 1, true, true);
+  V("Z6 128x128 t128 8x16 bk8 s6 minb2 ffma2", 128, 128, 8, 8, 16, 128, 6, 2, false, true);
+  V("Z7 128x256 t256 8x16 bk8 s4 minb1 ffma2", 128, 256, 8, 8, 16, 256, 4, 1, false, true);
+  V("Z8 64x128 t128 8x8 bk16 s3 minb2 ffma2", 64, 128, 16, 8, 8, 128, 3, 2, false, true);
+  V("Z9 128x128 t128 16x8 bk16 s3 minb2 ffma2", 128, 128, 16, 16, 8, 128, 3, 2, false, true);
+  V("Y10 64x128 t128 8x8 bk8 s4 minb3 ffma2", 64, 128, 8, 8, 8, 128, 4, 3, false, true);
+  V("Y11 64x128 t128 8x8 bk16 s4 minb3 ffma2", 64, 128, 16, 8, 8, 128, 4, 3, false, true);
+  V("Y12 64x128 t128 8x8 bk16 s3 minb2 db ffma2", 64, 128, 16, 8, 8, 128, 3, 2, true, true);
+  V("Y13 64x256 t256 8x8 bk16 s3 minb2 ffma2", 64, 256, 16, 8, 8, 256, 3, 2, false, true);
+  V("Y14 128x128 t256 8x8 bk16 s3 minb1 ffma2", 128, 128, 16, 8, 8, 256, 3, 1, false, true);
+  V("Y15 64x128 t128 8x8 bk32 s3 minb3 ffma2", 64, 128, 32, 8, 8, 128, 3, 3, false, true);
+  V("Y16 64x64 t64 8x8 bk16 s3 minb6 ffma2", 64, 64, 16, 8, 8, 64, 3, 6, false, true);
   return 0;
 }
