@@ -60,12 +60,6 @@ __global__ void __launch_bounds__(TTHREADS, tile_minb<SA, TC, TR, RD>()) tile_ke
   using RA = raw_t<SA>;
   constexpr int V = 16 / sizeof(RA);
   constexpr bool SAME = std::is_same<TC, TR>::value;
-  // paired f32 arithmetic (FFMA2 / FADD2); PS_TILE_SCALAR=1 at build time keeps scalar ops
-#ifdef PS_TILE_SCALAR
-  constexpr bool F2 = false;
-#else
-  constexpr bool F2 = std::is_same<TC, float>::value && std::is_same<TR, float>::value;
-#endif
   // rows per group: 16, or 8 where 16 would take more than 128 registers (2 CTAs per
   // SM instead of 1 keeps the same bytes in flight and fills all SMs; ptxas -v):
   // 16-bit chunks (V = 8) with row dots or an f64 compute type, f32 chunks (V = 4)
@@ -126,55 +120,6 @@ __global__ void __launch_bounds__(TTHREADS, tile_minb<SA, TC, TR, RD>()) tile_ke
           }
         }
         // 2) column-sum chains (i ascending) and lane row-dot chains (v ascending)
-        if constexpr (F2 && FULL) {
-          // f32 arithmetic on full groups: FFMA2 / FADD2 (two independent IEEE ops per
-          // instruction, so every chain is unchanged): column pairs (v, v+1) with w_i
-          // broadcast, row pairs (r, r+1) with x_v broadcast
-#pragma unroll
-          for (int r = 0; r < GR; r += 2) {
-            float a0[V], a1[V];
-#pragma unroll
-            for (int v = 0; v < V; v++) {
-              a0[v] = Ld<SA, float>::get(&ch[r].e[v], 0);
-              a1[v] = Ld<SA, float>::get(&ch[r + 1].e[v], 0);
-            }
-#pragma unroll
-            for (int h = 0; h < 2; h++) {
-              const float *av = h ? a1 : a0;
-              (void)av;   // CM_NONE: row dots only
-              if constexpr (CM == COL_DOT) {
-                const float wi = sw[g - i0 + r + h];
-#pragma unroll
-                for (int v = 0; v < V; v += 2) {
-                  const float2 t = __ffma2_rn(make_float2(av[v], av[v + 1]), make_float2(wi, wi),
-                                              make_float2(p[v], p[v + 1]));
-                  p[v] = t.x;
-                  p[v + 1] = t.y;
-                }
-              } else if constexpr (CM == COL_SUM) {
-#pragma unroll
-                for (int v = 0; v < V; v += 2) {
-                  const float2 t = __fadd2_rn(make_float2(p[v], p[v + 1]), make_float2(av[v], av[v + 1]));
-                  p[v] = t.x;
-                  p[v + 1] = t.y;
-                }
-              } else if constexpr (CM == COL_SQDEV) {
-#pragma unroll
-                for (int v = 0; v < V; v++) {
-                  const float d = av[v] - mu[v];
-                  p[v] = t_fma(d, d, p[v]);
-                }
-              }
-            }
-            if constexpr (RD) {
-              float2 l = make_float2(0.f, 0.f);
-#pragma unroll
-              for (int v = 0; v < V; v++) l = __ffma2_rn(make_float2(a0[v], a1[v]), make_float2(xv[v], xv[v]), l);
-              lp[r] = l.x;
-              lp[r + 1] = l.y;
-            }
-          }
-        } else {
 #pragma unroll
         for (int r = 0; r < GR; r++) {
           lp[r] = TR(0);
@@ -199,7 +144,6 @@ __global__ void __launch_bounds__(TTHREADS, tile_minb<SA, TC, TR, RD>()) tile_ke
               }
             }
           }
-        }
         }
       };
       if (wfull && nrow == GR) group(std::integral_constant<bool, true>());
