@@ -272,67 +272,6 @@ __device__ __forceinline__ void epi_chunk(const Params &p, float *stg, int lane,
   __syncwarp();
 }
 
-// Direct epilogue of one 32-row x 16-column chunk (PS_TC_EPI_DIRECT builds): lane =
-// row row0 + lane writes its 16 consecutive columns straight from registers as four
-// 16-byte (f32) / 8-byte (16-bit) accesses -- no shared-memory staging, which frees
-// 20 KiB for a seventh operand stage in the 2-CTA kernel.
-__device__ __forceinline__ void epi_chunk_direct(const Params &p, int lane, int64_t row0, int64_t col0,
-                                                 const uint32_t (&v)[16], int kab) {
-  const int64_t row = row0 + lane;
-  if (row >= p.M) return;
-  const bool vcol = p.vec4 && col0 + 15 < p.N;
-  const int64_t base = row * p.ldc + col0;
-  float c[16];
-#pragma unroll
-  for (int e = 0; e < 16; e++) c[e] = 0.f;
-  if (p.epi == EPI_AXPBY) {
-    if (vcol) {
-#pragma unroll
-      for (int q = 0; q < 4; q++) {
-        if (p.cin_type == PS_F32) {
-          const float4 t = __ldg(reinterpret_cast<const float4 *>((const float *)p.Cin + base) + q);
-          c[4 * q] = t.x; c[4 * q + 1] = t.y; c[4 * q + 2] = t.z; c[4 * q + 3] = t.w;
-        } else {
-          const uint2 t = __ldg(reinterpret_cast<const uint2 *>((const uint16_t *)p.Cin + base) + q);
-          const uint16_t h[4] = {(uint16_t)(t.x & 0xFFFF), (uint16_t)(t.x >> 16), (uint16_t)(t.y & 0xFFFF),
-                                 (uint16_t)(t.y >> 16)};
-#pragma unroll
-          for (int e = 0; e < 4; e++) c[4 * q + e] = p.cin_type == PS_BF16 ? bf16_to_f32(h[e]) : f16_to_f32(h[e]);
-        }
-      }
-    } else {
-#pragma unroll
-      for (int e = 0; e < 16; e++)
-        if (col0 + e < p.N) c[e] = load_c(p.Cin, p.cin_type, base + e);
-    }
-  }
-  float x[16];
-#pragma unroll
-  for (int e = 0; e < 16; e++) {
-    x[e] = __uint_as_float(v[e]);
-    if (kab) x[e] = scalbnf(x[e], kab);   // exact power-of-two scale (fp8)
-    x[e] = epi_op(p, x[e], c[e]);
-  }
-  if (vcol) {
-#pragma unroll
-    for (int q = 0; q < 4; q++) {
-      if (p.c_type == PS_F32) {
-        reinterpret_cast<float4 *>((float *)p.C + base)[q] = make_float4(x[4 * q], x[4 * q + 1], x[4 * q + 2], x[4 * q + 3]);
-      } else {
-        uint16_t h[4];
-#pragma unroll
-        for (int e = 0; e < 4; e++) h[e] = p.c_type == PS_BF16 ? rne_bf16(x[4 * q + e]) : rne_f16(x[4 * q + e]);
-        reinterpret_cast<uint2 *>((uint16_t *)p.C + base)[q] =
-            make_uint2((uint32_t)h[0] | ((uint32_t)h[1] << 16), (uint32_t)h[2] | ((uint32_t)h[3] << 16));
-      }
-    }
-  } else {
-#pragma unroll
-    for (int e = 0; e < 16; e++)
-      if (col0 + e < p.N) store_c(p.C, p.c_type, base + e, x[e]);
-  }
-}
-
 template <int ES>
 __global__ void __launch_bounds__(NTHREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
@@ -461,18 +400,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 // c, c + #clusters, ... (SYRK: lower tiles skipped by every role alike).
 namespace tc2 {
 
-#ifdef PS_TC_EPI_DIRECT
-constexpr int BM = 256, BN = 256, STAGES = 7;   // 7 x 32 KiB, epilogue straight from registers
-constexpr int EPI_BYTES = 0;
-#else
 constexpr int BM = 256, BN = 256, STAGES = 6;   // 6 x 32 KiB + 20 KiB epilogue staging
-constexpr int EPI_BYTES = tc::EPI_SMEM;
-#endif
 constexpr int HM = BM / 2, HN = BN / 2;          // per-CTA halves
 constexpr int A_BYTES = HM * tc::KB_BYTES;      // 16 KiB
 constexpr int B_BYTES = HN * tc::KB_BYTES;      // 16 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512 + EPI_BYTES;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 512 + tc::EPI_SMEM;
 constexpr int NTHREADS = tc::NTHREADS;
 constexpr uint32_t TMEM_COLS = 512;             // 2 accumulators x 256 f32 columns
 constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;     // shared::cluster address of the leader's copy
@@ -724,12 +657,7 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         if (pn0 + cc * EPI_COLS >= p.N) break;
         uint32_t v[16];
         tmem_ld16(tmem + acc * BN + ((uint32_t)(q * 32) << 16) + (uint32_t)(cc * EPI_COLS), v);
-#ifdef PS_TC_EPI_DIRECT
-        (void)stg;
-        tc::epi_chunk_direct(p, lane, row0, pn0 + cc * EPI_COLS, v, kab);
-#else
         epi_chunk(p, stg, lane, row0, pn0 + cc * EPI_COLS, v, kab);
-#endif
       }
       fence_before();
       __syncwarp();
