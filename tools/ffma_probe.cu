@@ -203,6 +203,126 @@ void run(const char *name, int n) {
   fflush(stdout);
 }
 
+
+// Variant family "K": A (k-major) lands by cp.async in its natural [m][k] layout
+// (row stride BK + 4 floats), no register staging and no transposed stores.  A
+// thread reads, per group of 4 k, one LDS.128 per owned row (4 k values) and two
+// LDS.128 of B per k; 8 x 8 outputs per thread as FFMA2 pairs along n.
+template <int BM, int BN, int BK, int THREADS, int S, int MINB>
+__global__ void __launch_bounds__(THREADS, MINB) ffma_kacp(const float *__restrict__ A, const float *__restrict__ B,
+                                                           float *__restrict__ C, int M, int N, int K) {
+  constexpr int TM = 8, TN = 8, TX = BN / TN, TY = BM / TM;
+  static_assert(TX * TY == THREADS, "grid");
+  constexpr int LA = BK + 4, LB = BN + 4;
+  constexpr int AEL = BM * LA, BEL = BK * LB;
+  extern __shared__ __align__(16) float sm[];
+  float *As0 = sm, *Bs0 = sm + S * AEL;
+  const int tid = threadIdx.x, tx = tid % TX, ty = tid / TX;
+  const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
+  const int ktiles = K / BK;
+  auto issue = [&](int kt, int st) {
+    float *As = As0 + st * AEL, *Bs = Bs0 + st * BEL;
+#pragma unroll
+    for (int c = tid; c < BM * BK / 4; c += THREADS) {
+      const int r = c / (BK / 4), kc = (c % (BK / 4)) * 4;
+      cp16(As + r * LA + kc, A + (size_t)(m0 + r) * K + kt * BK + kc);
+    }
+#pragma unroll
+    for (int c = tid; c < BK * BN / 4; c += THREADS) {
+      const int kr = c / (BN / 4), nc = (c % (BN / 4)) * 4;
+      cp16(Bs + kr * LB + nc, B + (size_t)(kt * BK + kr) * N + n0 + nc);
+    }
+  };
+  float2 acc[TM][TN / 2];
+#pragma unroll
+  for (int i = 0; i < TM; i++)
+#pragma unroll
+    for (int j = 0; j < TN / 2; j++) acc[i][j] = make_float2(0.f, 0.f);
+#pragma unroll
+  for (int s = 0; s < S - 1; s++) {
+    if (s < ktiles) issue(s, s);
+    commit();
+  }
+  for (int kt = 0; kt < ktiles; kt++) {
+    waitg<S - 2>();
+    __syncthreads();
+    const int nt = kt + S - 1;
+    if (nt < ktiles) issue(nt, nt % S);
+    commit();
+    const float *As = As0 + (kt % S) * AEL, *Bs = Bs0 + (kt % S) * BEL;
+#pragma unroll
+    for (int k4 = 0; k4 < BK; k4 += 4) {
+      float4 a[TM];
+#pragma unroll
+      for (int i = 0; i < TM; i++)
+        a[i] = *reinterpret_cast<const float4 *>(As + ((i / 4) * TY * 4 + ty * 4 + (i % 4)) * LA + k4);
+#pragma unroll
+      for (int kk = 0; kk < 4; kk++) {
+        const float4 b0 = *reinterpret_cast<const float4 *>(Bs + (k4 + kk) * LB + tx * 4);
+        const float4 b1 = *reinterpret_cast<const float4 *>(Bs + (k4 + kk) * LB + TX * 4 + tx * 4);
+        const float2 b[4] = {make_float2(b0.x, b0.y), make_float2(b0.z, b0.w), make_float2(b1.x, b1.y),
+                             make_float2(b1.z, b1.w)};
+#pragma unroll
+        for (int i = 0; i < TM; i++) {
+          const float ai = kk == 0 ? a[i].x : kk == 1 ? a[i].y : kk == 2 ? a[i].z : a[i].w;
+#pragma unroll
+          for (int j = 0; j < TN / 2; j++) acc[i][j] = __ffma2_rn(make_float2(ai, ai), b[j], acc[i][j]);
+        }
+      }
+    }
+  }
+  waitg<0>();
+#pragma unroll
+  for (int i = 0; i < TM; i++) {
+    const int gm = m0 + (i / 4) * TY * 4 + ty * 4 + (i % 4);
+#pragma unroll
+    for (int j4 = 0; j4 < TN / 4; j4++) {
+      const int gn = n0 + j4 * TX * 4 + tx * 4;
+      *reinterpret_cast<float4 *>(C + (size_t)gm * N + gn) =
+          make_float4(acc[i][j4 * 2].x, acc[i][j4 * 2].y, acc[i][j4 * 2 + 1].x, acc[i][j4 * 2 + 1].y);
+    }
+  }
+}
+
+template <int BM, int BN, int BK, int THREADS, int S, int MINB>
+void run_kacp(const char *name, int n) {
+  auto k = ffma_kacp<BM, BN, BK, THREADS, S, MINB>;
+  const int smem = S * (BM * (BK + 4) + BK * (BN + 4)) * 4;
+  CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  cudaFuncAttributes fa;
+  CK(cudaFuncGetAttributes(&fa, k));
+  int occ = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, THREADS, smem));
+  const int c = 1024;
+  k<<<dim3(c / BN, c / BM), THREADS, smem>>>(dA, dB, dC, c, c, c);
+  ref_kernel<<<dim3(c / 256, c), 256>>>(dA, dB, dR, c, c, c);
+  CK(cudaDeviceSynchronize());
+  std::vector<uint32_t> h1((size_t)c * c), h2((size_t)c * c);
+  CK(cudaMemcpy(h1.data(), dC, h1.size() * 4, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(h2.data(), dR, h2.size() * 4, cudaMemcpyDeviceToHost));
+  size_t bad = 0;
+  for (size_t i = 0; i < h1.size(); i++) bad += h1[i] != h2[i];
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  dim3 g(n / BN, n / BM);
+  k<<<g, THREADS, smem>>>(dA, dB, dC, n, n, n);
+  float best = 1e30f;
+  for (int r = 0; r < 5; r++) {
+    cudaEventRecord(e0);
+    k<<<g, THREADS, smem>>>(dA, dB, dC, n, n, n);
+    cudaEventRecord(e1);
+    CK(cudaEventSynchronize(e1));
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms < best) best = ms;
+  }
+  printf("{\"variant\": \"%s\", \"regs\": %d, \"smem\": %d, \"ctas_per_sm\": %d, \"mismatch_1024\": %zu, \"N\": %d, "
+         "\"ms\": %.3f, \"tflops\": %.1f}\n",
+         name, fa.numRegs, smem, occ, bad, n, best, 2.0 * n * n * (double)n / (best * 1e-3) / 1e12);
+  fflush(stdout);
+}
+
 __global__ void fill(float *p, size_t n, uint32_t seed) {
   size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
   if (i < n) {
@@ -256,5 +376,13 @@ int main(int argc, char **argv) {
   V("Y14 128x128 t256 8x8 bk16 s3 minb1 ffma2", 128, 128, 16, 8, 8, 256, 3, 1, false, true);
   V("Y15 64x128 t128 8x8 bk32 s3 minb3 ffma2", 64, 128, 32, 8, 8, 128, 3, 3, false, true);
   V("Y16 64x64 t64 8x8 bk16 s3 minb6 ffma2", 64, 64, 16, 8, 8, 64, 3, 6, false, true);
+#define VK(name, ...) if (!*only || strstr(name, only)) run_kacp<__VA_ARGS__>(name, n)
+  VK("K1 acp 64x128 t128 bk16 s3 minb3", 64, 128, 16, 128, 3, 3);
+  VK("K2 acp 64x128 t128 bk16 s4 minb3", 64, 128, 16, 128, 4, 3);
+  VK("K3 acp 64x128 t128 bk32 s3 minb2", 64, 128, 32, 128, 3, 2);
+  VK("K4 acp 128x128 t256 bk16 s3 minb2", 128, 128, 16, 256, 3, 2);
+  VK("K5 acp 128x128 t256 bk16 s4 minb1", 128, 128, 16, 256, 4, 1);
+  VK("K6 acp 128x64 t128 bk16 s4 minb2", 128, 64, 16, 128, 4, 2);
+  VK("K7 acp 64x128 t128 bk8 s6 minb3", 64, 128, 8, 128, 6, 3);
   return 0;
 }
