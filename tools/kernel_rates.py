@@ -69,6 +69,10 @@ if "tc" in WHICH:    # tcgen05: fp16, bf16, e4m3, e5m2 multiplicands, f32 C
     lib_rate("gemm", [3, 3, 1], B.FLAG_BF16, gemm, "gemm_tc2_kernel bf16")
     lib_rate("gemm", [4, 4, 1], B.FLAG_FP8, gemm, "gemm_tc2_kernel e4m3")
     lib_rate("gemm", [5, 5, 1], B.FLAG_FP8, gemm, "gemm_tc2_kernel e5m2")
+if "tcaxpby" in WHICH:   # alpha/beta GEMM with a 16-bit C (Cin read + C write in fp16 / bf16),
+    # the same operation as cuBLAS addmm(beta, C, alpha, A, B) below
+    lib_rate("gemm", [2, 2, 2], 0, gemm, "gemm_tc2_kernel fp16, alpha/beta epilogue, C fp16")
+    lib_rate("gemm", [3, 3, 3], B.FLAG_BF16, gemm, "gemm_tc2_kernel bf16, alpha/beta epilogue, C bf16")
 if "cublas" in WHICH:
     def tm(f, reps=10):
         f()
@@ -88,6 +92,14 @@ if "cublas" in WHICH:
         ms = tm(lambda: a @ b)
         emit(kernel="cuBLAS matmul", dtype=str(dt), N=N, kernel_ms=round(ms, 4), tflops=round(gemm / (ms * 1e-3) / 1e12, 1))
         del a, b
+    for dt in (torch.float16, torch.bfloat16):   # C <- beta C + alpha A B, 16-bit C read and written
+        a = torch.randn(N, N, device="cuda").to(dt)
+        b = torch.randn(N, N, device="cuda").to(dt)
+        c = torch.randn(N, N, device="cuda").to(dt)
+        ms = tm(lambda: torch.addmm(c, a, b, beta=0.5, alpha=1.5))
+        emit(kernel="cuBLAS addmm (beta C + alpha A B)", dtype=str(dt), N=N, kernel_ms=round(ms, 4),
+             tflops=round(gemm / (ms * 1e-3) / 1e12, 1))
+        del a, b, c
     # f32 with TF32 off: cuBLAS's own FFMA SGEMM, the practical ceiling for gemm_ffma_kernel
     torch.backends.cuda.matmul.allow_tf32 = False
     a = torch.randn(N, N, device="cuda")
