@@ -45,14 +45,15 @@ struct TileArgs {
 };
 
 // Minimum CTAs per SM for __launch_bounds__: 16-bit A with f32 arithmetic and row
-// dots (8-row groups) is capped at 80 registers so THREE CTAs share an SM -- these
-// statements are bound by global-load latency (ncu: long_scoreboard 57% of stalls,
-// 14 of 64 warps active), so 50% more warps in flight is what they need.  0 = not
-// specified (ptxas keeps its default, <= 128 registers here; an explicit 1 lets it
-// grow to ~230 and halves the occupancy of the f64 statements)
+// dots runs 16-row groups capped at 128 registers, two CTAs per SM -- these statements
+// are bound by global-load latency (ncu: long_scoreboard 57% of stalls), and twice the
+// rows in flight per warp beat 50% more warps: 8-row groups at 80 registers and three
+// CTAs per SM measured 4.5-7.6% slower (profiles/tile_probe_{base,gr16}_r2as.jsonl).
+// 0 = not specified (ptxas keeps its default, <= 128 registers here; an explicit 1
+// lets it grow to ~230 and halves the occupancy of the f64 statements)
 template <class SA, class TC, class TR, bool RD>
 constexpr int tile_minb() {
-  return (RD && sizeof(raw_t<SA>) == 2 && sizeof(TC) == 4 && sizeof(TR) == 4) ? 3 : 0;
+  return (RD && sizeof(raw_t<SA>) == 2 && sizeof(TC) == 4 && sizeof(TR) == 4) ? 2 : 0;
 }
 
 template <class SA, class TC, class TR, int CM, bool RD>
@@ -62,9 +63,9 @@ __global__ void __launch_bounds__(TTHREADS, tile_minb<SA, TC, TR, RD>()) tile_ke
   constexpr bool SAME = std::is_same<TC, TR>::value;
   // rows per group: 16, or 8 where 16 would take more than 128 registers (2 CTAs per
   // SM instead of 1 keeps the same bytes in flight and fills all SMs; ptxas -v):
-  // 16-bit chunks (V = 8) with row dots or an f64 compute type, f32 chunks (V = 4)
-  // feeding f64 column sums or weighted (COL_DOT) f32 column sums without row dots
-  constexpr int GR = ((V == 8 && (RD || sizeof(TC) == 8 || sizeof(TR) == 8)) ||
+  // 16-bit chunks (V = 8) with an f64 compute type, f32 chunks (V = 4) feeding f64
+  // column sums or weighted (COL_DOT) f32 column sums without row dots
+  constexpr int GR = ((V == 8 && (sizeof(TC) == 8 || sizeof(TR) == 8)) ||
                       (V == 4 && !RD && (CM == COL_DOT || sizeof(TC) == 8)))
                          ? 8
                          : 16;
