@@ -31,12 +31,13 @@ constexpr int64_t FGROUP_M = 16;
 constexpr int FTM = 8, FTN = 8, FTX = FBN / FTN, FTY = FBM / FTM;   // 16 x 8 threads
 constexpr int FLA = FBM + FPAD, FLB = FBN + FPAD;   // row strides of As[k][m], Bs[k][n]
 // k-tile depth and ring length per operand types (measured at 8192^3, profiles/
-// kernel_rates_ffma2_r2ad.jsonl vs r2ac): BK = 16 x 3 stages for 16-bit A with f32 B
-// (55.2 vs 51.2 TFLOP/s), BK = 8 x 4 stages otherwise (f32 52.8 vs 51.5, 16-bit B
-// 51.6 vs 48.2): the shallower tile halves the register-staged run per thread
+// kernel_rates_ffma2_r2ad.jsonl vs r2ac, ffma_tile_*_r2aw.jsonl): BK = 16 x 3 stages for
+// 16-bit A with f32 B (55.3 vs 51.2 TFLOP/s at BK = 8), BK = 8 x 6 stages otherwise
+// (f32 53.3, 16-bit B 53.1; x 4 stages 52.8 / 51.6; BK = 16: 51.5 / 48.2): the shallower
+// tile halves the register-staged run per thread, the longer ring covers its latency
 template <class SA, class SB> struct FTile {
   static constexpr bool DEEP = !std::is_same<SA, float>::value && std::is_same<SB, float>::value;
-  static constexpr int BK = DEEP ? 16 : 8, S = DEEP ? 3 : 4;
+  static constexpr int BK = DEEP ? 16 : 8, S = DEEP ? 3 : 6;
   static constexpr int A_EL = BK * FLA, B_EL = BK * FLB;
   static constexpr int SMEM = S * (A_EL + B_EL) * 4;
 };

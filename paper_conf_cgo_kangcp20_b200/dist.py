@@ -30,10 +30,10 @@ F64, F32, F16, BF16, E4M3, E5M2 = 0, 1, 2, 3, 4, 5
 SIZE = {F64: 8, F32: 4, F16: 2, BF16: 2, E4M3: 1, E5M2: 1}
 FP8 = (E4M3, E5M2)
 # B200 rates for the cost model, as measured by this library's kernels at 8192^3
-# (conversion ~6.5 TB/s, f64 DMMA 34.2, f32 FFMA2 52.8, tcgen05 fp16
+# (conversion ~6.5 TB/s, f64 DMMA 34.2, f32 FFMA2 53.3, tcgen05 fp16
 # 1461 and fp8 2796 TFLOP/s); only relative values matter for the partition
 HBM_BPS = 6.5e12
-PEAK = {"tc": 1.46e15, "tc8": 2.8e15, F32: 52.8e12, F64: 34.2e12}
+PEAK = {"tc": 1.46e15, "tc8": 2.8e15, F32: 53.3e12, F64: 34.2e12}
 
 # statement tables: ("mv", A, [objects]) = one streaming pass over object A;
 # ("mm", a, b, out, (M, N, K)) = contraction; ("ew", [objects]) = elementwise
